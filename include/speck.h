@@ -1,0 +1,189 @@
+/*
+ * speck.h — C ABI of the B200-native spECK SpGEMM library (libspeck.so).
+ *
+ * Computes C = A·B for sparse matrices in CSR format (Parger et al., PPoPP'20; citations
+ * "P:a-b" are lines of the paper text PAPER.md):
+ *   C_ij = Σ_k A_ik · B_kj                                   eq. (1)
+ * CSR stores "the NZ elements sorted row-major and column-minor ... a sorted array of
+ * row offsets indicates the beginning of each row".  The output C is sorted
+ * CSR as well.  Every stored (structural) product counts:
+ * entries whose value cancels to 0.0 are kept (the symbolic pass counts "without
+ * calculating their values"; reading R1).
+ *
+ * The call sequence follows the paper's pipeline (Fig. 2):
+ *   speck_analyze  = row analysis (Alg. 1) -> symbolic global load balancing
+ *                     -> symbolic SpGEMM -> prefix sum of the
+ *                    row sizes.  Returns nnz(C); the CALLER allocates C
+ *                    (allocation of C is outside the paper's timing).
+ *   speck_spgemm   = numeric global load balancing -> numeric SpGEMM with
+ *                    direct / hash / dense accumulators and in-scratchpad sorting
+ *                    (P:1121-1148).
+ *
+ * Conventions (all functions):
+ *   - Matrix pointers are DEVICE pointers on the handle's device.  row_ptr is int64
+ *     [rows+1] with row_ptr[0] == 0, col_idx is int32 [nnz], values fp32 or fp64 [nnz].
+ *     A, B and C share one value type.
+ *   - Inputs are borrowed and never written; C arrays are caller-owned.  Workspace is
+ *     owned by the handle, grown on demand and reused across calls; speck_destroy frees it.
+ *   - Work is issued on the caller's `stream` (0 = legacy default stream).  The library
+ *     forks internal streams for concurrent kernels and joins them back onto `stream`.
+ *   - No exception crosses the ABI.  Every function returns a speck_status_t; the text of
+ *     the last error of a handle is available from speck_last_error().
+ *   - A handle is bound to one device and is not thread-safe.
+ *   - Input rows must be sorted with unique columns.  Unsorted or duplicate
+ *     columns are undefined behaviour unless SPECK_OPT_VALIDATE is set, which turns them
+ *     into SPECK_ERR_INVALID_INPUT.
+ *   - Column indices must be < 2^31 - 1.  nnz(C) and per-matrix nnz are int64.
+ */
+#ifndef SPECK_H_
+#define SPECK_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct speck_handle_s* speck_handle_t;
+typedef void* speck_stream_t; /* a cudaStream_t */
+
+typedef enum {
+  SPECK_OK = 0,
+  SPECK_ERR_INVALID_ARGUMENT = 1,  /* null pointer with nnz > 0, negative dims, bad option */
+  SPECK_ERR_DIMENSION_MISMATCH = 2,/* A.cols != B.rows */
+  SPECK_ERR_DTYPE_MISMATCH = 3,    /* A and B value types differ */
+  SPECK_ERR_UNSUPPORTED = 4,       /* e.g. cols >= 2^31 - 1 */
+  SPECK_ERR_OUT_OF_MEMORY = 5,     /* workspace allocation failed */
+  SPECK_ERR_CUDA = 6,              /* any CUDA runtime / launch error; see speck_last_error */
+  SPECK_ERR_NOT_ANALYZED = 7,      /* speck_spgemm without a matching speck_analyze */
+  SPECK_ERR_INVALID_INPUT = 8      /* validation (SPECK_OPT_VALIDATE) found unsorted/duplicate/out-of-range columns */
+} speck_status_t;
+
+typedef enum { SPECK_F32 = 0, SPECK_F64 = 1 } speck_dtype_t;
+
+/* A borrowed CSR matrix.  values may be NULL for speck_analyze /
+ * speck_row_analysis (structure only). */
+typedef struct {
+  int64_t rows;
+  int64_t cols;
+  int64_t nnz;
+  const int64_t* row_ptr; /* device, [rows+1] */
+  const int32_t* col_idx; /* device, [nnz], sorted ascending per row */
+  const void* values;     /* device, [nnz] fp32 or fp64 */
+  speck_dtype_t dtype;
+} speck_csr_t;
+
+/* Options (speck_set_option).  Defaults in brackets.  All are plan/test knobs: none of
+ * them changes the result, only which accumulator / load-balancing path produces it. */
+typedef enum {
+  SPECK_OPT_GLOBAL_LB_SYMBOLIC = 0, /* -1 auto by Table 2 thresholds, 0 off, 1 on [-1] */
+  SPECK_OPT_GLOBAL_LB_NUMERIC = 1,  /* same for the numeric step [-1] */
+  SPECK_OPT_FORCE_ACCUMULATOR = 2,  /* 0 auto; 1 hash wherever it fits; 2 dense for every non-direct row [0] */
+  SPECK_OPT_DENSE_WINDOW = 3,       /* >0: cap the dense accumulator window (columns) — Fig. 5 tests [0] */
+  SPECK_OPT_STAGE_TIMING = 4,       /* 1: record per-stage times with CUDA events (syncs) [0] */
+  SPECK_OPT_VALIDATE = 5,           /* 1: validate input CSR (sorted, unique, in range) [0] */
+  SPECK_OPT_DISABLE_DIRECT = 6,     /* 1: route single-NZ rows through the accumulators [0] */
+  SPECK_OPT_FIXED_GROUP_SIZE = 7,   /* >0: use this g for every block instead of the local LB [0] */
+  SPECK_OPT_CONCURRENT_STREAMS = 8  /* number of internal streams for concurrent bins, 1..8 [4] */
+} speck_option_t;
+
+/* Statistics of the last analyze/spgemm pair (speck_get_stats). */
+typedef struct {
+  int64_t products;          /* Σ_i prods_i (Alg. 1 line 10); FLOP = 2·products */
+  int64_t max_row_products;  /* prod_max (Alg. 1 line 11) */
+  int64_t nnz_c;             /* nnz(C) */
+  int64_t rows_direct;       /* rows with a single NZ in A */
+  int64_t rows_empty;        /* rows without products */
+  int32_t lb_symbolic;       /* 1 if the global load balancer ran for the symbolic step */
+  int32_t lb_numeric;        /* 1 if it ran for the numeric step */
+  int64_t rows_per_bin_symbolic[8]; /* [0]=empty [1]=direct [2..6]=configs 0..4 (cfg 4 incl. dense) [7]=dense */
+  int64_t rows_per_bin_numeric[8];
+  int64_t rows_dense_numeric;    /* rows accumulated with the dense accumulator in the numeric step */
+  int64_t workspace_bytes;       /* workspace currently held by the handle */
+  int64_t kernel_launches;       /* kernels this handle has launched since speck_create (cumulative) */
+  float ms_analysis, ms_symbolic_lb, ms_symbolic, ms_scan, ms_numeric_lb, ms_numeric; /* SPECK_OPT_STAGE_TIMING */
+} speck_stats_t;
+
+/* Create a handle on `device` (CUDA ordinal). */
+speck_status_t speck_create(speck_handle_t* handle, int device);
+
+/* Release all workspace and the handle.  Synchronises the handle's device. */
+speck_status_t speck_destroy(speck_handle_t handle);
+
+/* Set a plan option (speck_option_t). */
+speck_status_t speck_set_option(speck_handle_t handle, int option, int64_t value);
+
+/* Symbolic phase: rows analysis (Alg. 1), global load balancing, symbolic SpGEMM and the
+ * exclusive prefix sum of the C row sizes.
+ *   C_row_ptr : device int64 [A.rows + 1], caller-owned, written with C's row offsets
+ *   nnz_c     : host out, nnz(C) = C_row_ptr[A.rows]
+ * Synchronises `stream` twice (the analysis statistics and nnz(C) are read back).
+ * A.values / B.values are not read. */
+speck_status_t speck_analyze(speck_handle_t handle, const speck_csr_t* A, const speck_csr_t* B,
+                             int64_t* C_row_ptr, int64_t* nnz_c, speck_stream_t stream);
+
+/* Numeric phase: writes C_col_idx [nnz_c] and C_values [nnz_c] (caller-allocated, device)
+ * for the A, B of the preceding speck_analyze on this handle (same pointers and shapes,
+ * else SPECK_ERR_NOT_ANALYZED).  Rows come out sorted by column.  Asynchronous. */
+speck_status_t speck_spgemm(speck_handle_t handle, const speck_csr_t* A, const speck_csr_t* B,
+                            const int64_t* C_row_ptr, int32_t* C_col_idx, void* C_values,
+                            speck_stream_t stream);
+
+/* Row analysis only (Alg. 1).  Per row i of A (device arrays, [A.rows]):
+ *   prods[i]  = Σ_{k ∈ A_i} |B_k|           maxlen[i] = max_k |B_k|
+ *   colmin[i] = min over non-empty B_k of the first column (INT32_MAX if none)
+ *   colmax[i] = max over non-empty B_k of the last column  (-1 if none)
+ * Any output pointer may be NULL.  Used by the multi-GPU row partitioner (balanced
+ * product split).  Asynchronous. */
+speck_status_t speck_row_analysis(speck_handle_t handle, const speck_csr_t* A, const speck_csr_t* B,
+                                  int64_t* prods, int32_t* maxlen, int32_t* colmin, int32_t* colmax,
+                                  speck_stream_t stream);
+
+/* Statistics of the last analyze/spgemm (host struct). */
+speck_status_t speck_get_stats(speck_handle_t handle, speck_stats_t* out);
+
+/* Static text for a status code. */
+const char* speck_status_string(speck_status_t status);
+
+/* Detail text of the last error on this handle ("" if none).  Valid until the next call. */
+const char* speck_last_error(speck_handle_t handle);
+
+/* Library version string. */
+const char* speck_version(void);
+
+/* ----------------------------------------------------------------------------------
+ * Component entry points.  They run the SAME device functions the pipeline uses, on
+ * device buffers, so the paper's worked examples and the plan logic can be checked
+ * against the oracle in isolation.  All asynchronous on `stream`.
+ * ---------------------------------------------------------------------------------- */
+
+/* Block merge (Alg. 2; Fig. 3), reading R10: for each aligned group
+ * of 32 entries of needs[n] (int64, device), neighbouring blocks are merged level by level
+ * (5 levels) while their sum stays strictly below `cap`.  Writes block_start_flag[n]
+ * (uint8, device): 1 where a block starts. */
+speck_status_t speck_block_merge(speck_handle_t handle, const int64_t* needs, int64_t n, int64_t cap,
+                                 uint8_t* block_start_flag, speck_stream_t stream);
+
+/* Local load balancer group size g (reading R9) for n blocks described by
+ * device arrays nnzA[n], prods[n], maxlen[n] (int64) and T threads; writes g[n] (int32). */
+speck_status_t speck_group_size(speck_handle_t handle, int32_t T, const int64_t* nnzA, const int64_t* prods,
+                                const int64_t* maxlen, int64_t n, int32_t* g, speck_stream_t stream);
+
+/* Scratchpad linear-probing hash (Fig. 4) with injected home slots: inserts
+ * keys[n] (uint32, device) at homes[n] (uint32) into a map of `size` slots (<= 8192) held
+ * in shared memory by one CTA, counting duplicates; copies the map out to
+ * slot_keys[size] (uint32, 0xFFFFFFFF = empty) and slot_counts[size] (uint32).
+ * Inserts are issued in order (one thread) so the final layout is deterministic. */
+speck_status_t speck_hash_probe(speck_handle_t handle, const uint32_t* keys, const uint32_t* homes, int64_t n,
+                                int32_t size, uint32_t* slot_keys, uint32_t* slot_counts, speck_stream_t stream);
+
+/* Exclusive prefix sum of int64 in[n] into out[n+1] (out[n] = total) with the library's
+ * single-pass decoupled look-back scan (the C row-offset step). */
+speck_status_t speck_exclusive_scan(speck_handle_t handle, const int64_t* in, int64_t n, int64_t* out,
+                                    speck_stream_t stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SPECK_H_ */

@@ -291,11 +291,12 @@ int64_t oracle_group_iters(int64_t nrows, const int64_t *lens, int64_t T, int64_
 }
 
 static int64_t round_pow2(double x) {
-    /* nearest power of two in log2 space ("round g to the closest power of two") */
+    /* "we also round g to the closest power of two": of the two powers of two
+     * p <= x < 2p, the one at the smaller |x - p| distance; a tie goes to 2p (reading R9). */
     if (x <= 1.0) return 1;
-    double l = log2(x);
-    int64_t e = (int64_t)floor(l + 0.5);
-    return (int64_t)1 << e;
+    int64_t p = 1;
+    while ((double)(2 * p) <= x) p *= 2;
+    return (x - (double)p < (double)(2 * p) - x) ? p : 2 * p;
 }
 
 /* Local load balancer, reading R9:

@@ -1,0 +1,790 @@
+// speck_api.cu — C ABI (include/speck.h), handle/workspace management and the host-side
+// plan of the spECK pipeline (Fig. 2) on B200.
+//
+// Host decisions follow §5: the global load balancer runs for a step when
+// m_max/m_avg and rows_C exceed the Table 2 thresholds, with the "*" set when
+// the longest row needs one of the largest kernels; otherwise rows are processed in fixed
+// groups of consecutive rows by one configuration big enough for the longest row
+// (P:806-818).
+#include <algorithm>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "plan_kernels.cuh"
+#include "spgemm_kernels.cuh"
+
+#define SPECK_VERSION "speck-b200 0.1.0 (sm_100a)"
+
+namespace speck {
+
+// Table 2 thresholds: {ratio, rows} for all kernels and for the largest ones.
+struct LbThresholds { double ratio, rows, ratio_big, rows_big; int big_from_cfg; };
+static const LbThresholds kLbSym = {39.2, 28000, 6.0, 5431, 2};  // "*" = three largest (caption, reading R11)
+static const LbThresholds kLbNum = {10.5, 23006, 1.3, 1238, 3};  // "*" = two largest
+
+struct Buf {
+  void* p = nullptr;
+  size_t cap = 0;
+};
+
+}  // namespace speck
+
+using namespace speck;
+
+struct speck_handle_s {
+  int device = 0;
+  int num_sms = 148;
+  std::string err;
+  // options
+  int64_t opt_lb_sym = -1, opt_lb_num = -1, opt_force_acc = 0, opt_dense_window = 0, opt_timing = 0, opt_validate = 0,
+          opt_disable_direct = 0, opt_fixed_g = 0, opt_streams = 4;
+  // workspace
+  Buf prods, maxlen, colmin, colmax, cnt, hist, hist_off, bins, stats, scan_status, resume, small;
+  unsigned long long* h_pinned = nullptr;  // pinned readback area (64 x u64)
+  cudaStream_t streams[kMaxStreams] = {};
+  cudaEvent_t ev_fork = nullptr, ev_join[kMaxStreams] = {};
+  cudaEvent_t ev_t[8] = {};
+  // plan state of the last analyze
+  bool analyzed = false;
+  const int64_t* A_rp = nullptr; const int32_t* A_col = nullptr; int64_t A_rows = 0, A_cols = 0, A_nnz = 0;
+  const int64_t* B_rp = nullptr; const int32_t* B_col = nullptr; int64_t B_rows = 0, B_cols = 0, B_nnz = 0;
+  speck_dtype_t dtype = SPECK_F32;
+  int64_t nnz_c = 0, max_cnt = 0, max_nnza = 0;
+  int64_t num_cat_start[CAT_COUNT + 1] = {};
+  speck_stats_t st = {};
+  int lb_num = 0;
+  bool numeric_pending = false;
+  int64_t launches = 0;  // kernels launched by this handle (cumulative)
+};
+
+namespace {
+
+speck_status_t fail(speck_handle_t h, speck_status_t s, const char* fmt, ...) {
+  if (h) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    h->err = buf;
+  }
+  return s;
+}
+
+#define CK(call)                                                                                      \
+  do {                                                                                                \
+    cudaError_t e_ = (call);                                                                          \
+    if (e_ != cudaSuccess)                                                                            \
+      return fail(h, e_ == cudaErrorMemoryAllocation ? SPECK_ERR_OUT_OF_MEMORY : SPECK_ERR_CUDA,      \
+                  "%s failed: %s (%s:%d)", #call, cudaGetErrorString(e_), __FILE__, __LINE__);        \
+  } while (0)
+
+#define CKL()                                                                                         \
+  do {                                                                                                \
+    ++h->launches;                                                                                    \
+    cudaError_t e_ = cudaGetLastError();                                                              \
+    if (e_ != cudaSuccess)                                                                            \
+      return fail(h, SPECK_ERR_CUDA, "kernel launch failed: %s (%s:%d)", cudaGetErrorString(e_),      \
+                  __FILE__, __LINE__);                                                                \
+  } while (0)
+
+speck_status_t ensure(speck_handle_t h, Buf& b, size_t bytes, cudaStream_t s) {
+  if (bytes <= b.cap) return SPECK_OK;
+  if (b.p) CK(cudaFreeAsync(b.p, s));
+  b.p = nullptr;
+  b.cap = 0;
+  size_t want = std::max<size_t>(bytes + bytes / 4, 4096);
+  cudaError_t e = cudaMallocAsync(&b.p, want, s);
+  if (e != cudaSuccess) {
+    (void)cudaGetLastError();
+    return fail(h, SPECK_ERR_OUT_OF_MEMORY, "workspace allocation of %zu bytes failed: %s", want,
+                cudaGetErrorString(e));
+  }
+  b.cap = want;
+  return SPECK_OK;
+}
+
+int64_t ws_bytes(speck_handle_t h) {
+  return (int64_t)(h->prods.cap + h->maxlen.cap + h->colmin.cap + h->colmax.cap + h->cnt.cap + h->hist.cap +
+                   h->hist_off.cap + h->bins.cap + h->stats.cap + h->scan_status.cap + h->resume.cap + h->small.cap);
+}
+
+speck_status_t check_csr(speck_handle_t h, const speck_csr_t* M, const char* name, bool need_values) {
+  if (!M) return fail(h, SPECK_ERR_INVALID_ARGUMENT, "%s is NULL", name);
+  if (M->rows < 0 || M->cols < 0 || M->nnz < 0) return fail(h, SPECK_ERR_INVALID_ARGUMENT, "%s has negative dims", name);
+  if (M->cols >= 0x7fffffffLL || M->rows >= 0x7fffffffLL)
+    return fail(h, SPECK_ERR_UNSUPPORTED, "%s: rows/cols must be < 2^31-1", name);
+  if (!M->row_ptr && M->rows > 0) return fail(h, SPECK_ERR_INVALID_ARGUMENT, "%s.row_ptr is NULL", name);
+  if (M->nnz > 0 && !M->col_idx) return fail(h, SPECK_ERR_INVALID_ARGUMENT, "%s.col_idx is NULL", name);
+  if (need_values && M->nnz > 0 && !M->values) return fail(h, SPECK_ERR_INVALID_ARGUMENT, "%s.values is NULL", name);
+  if (M->dtype != SPECK_F32 && M->dtype != SPECK_F64) return fail(h, SPECK_ERR_INVALID_ARGUMENT, "%s.dtype invalid", name);
+  return SPECK_OK;
+}
+
+template <typename F>
+speck_status_t launch_analysis(speck_handle_t h, int ga, F&& f) {
+  switch (ga) {
+    case 1: f(k_analysis<1>); break;
+    case 2: f(k_analysis<2>); break;
+    case 4: f(k_analysis<4>); break;
+    case 8: f(k_analysis<8>); break;
+    case 16: f(k_analysis<16>); break;
+    default: f(k_analysis<32>); break;
+  }
+  CKL();
+  return SPECK_OK;
+}
+
+int pow2_clamp(double x, int lo, int hi) {
+  int p = lo;
+  while (p * 2 <= hi && (double)(p * 2) <= x) p *= 2;
+  return p;
+}
+
+// kernel function pointer for (cfg, pass, V)
+template <typename V>
+void* spgemm_fn(int cfg, int pass) {
+  switch (cfg * 2 + pass) {
+    case 0: return (void*)k_spgemm<0, 0, V>;
+    case 1: return (void*)k_spgemm<0, 1, V>;
+    case 2: return (void*)k_spgemm<1, 0, V>;
+    case 3: return (void*)k_spgemm<1, 1, V>;
+    case 4: return (void*)k_spgemm<2, 0, V>;
+    case 5: return (void*)k_spgemm<2, 1, V>;
+    case 6: return (void*)k_spgemm<3, 0, V>;
+    case 7: return (void*)k_spgemm<3, 1, V>;
+    case 8: return (void*)k_spgemm<4, 0, V>;
+    default: return (void*)k_spgemm<4, 1, V>;
+  }
+}
+
+template <typename V>
+speck_status_t launch_spgemm(speck_handle_t h, int cfg, int pass, const SpgemmArgs<V>& a, cudaStream_t s) {
+  if (a.n_entries <= 0) return SPECK_OK;
+  const int64_t grid = (a.n_entries + a.group_rows - 1) / a.group_rows;
+  void* fn = spgemm_fn<V>(cfg, pass);
+  void* args[] = {(void*)&a};
+  CK(cudaLaunchKernel(fn, dim3((unsigned)grid), dim3(kCfgThreads[cfg]), args, (size_t)kCfgMapBytes[cfg], s));
+  ++h->launches;
+  return SPECK_OK;
+}
+
+template <typename V>
+speck_status_t set_smem_attrs(speck_handle_t h) {
+  for (int c = 0; c < kNumCfg; ++c)
+    for (int pass = 0; pass < 2; ++pass)
+      CK(cudaFuncSetAttribute(spgemm_fn<V>(c, pass), cudaFuncAttributeMaxDynamicSharedMemorySize, kCfgMapBytes[c]));
+  return SPECK_OK;
+}
+
+speck_status_t launch_scan(speck_handle_t h, const int64_t* in, int64_t n, int64_t* out, unsigned long long* max_out,
+                           cudaStream_t s) {
+  const int64_t tiles = n / kScanTile + 1;
+  speck_status_t st = ensure(h, h->scan_status, (size_t)tiles * 8 + 64, s);
+  if (st) return st;
+  CK(cudaMemsetAsync(h->scan_status.p, 0, (size_t)tiles * 8 + 64, s));
+  unsigned int* counter = reinterpret_cast<unsigned int*>(static_cast<char*>(h->scan_status.p) + tiles * 8);
+  k_scan<<<(unsigned)tiles, kScanThreads, 0, s>>>(in, n, out, static_cast<unsigned long long*>(h->scan_status.p), counter,
+                                                 max_out);
+  CKL();
+  return SPECK_OK;
+}
+
+// fork: internal streams wait for the user stream
+speck_status_t fork(speck_handle_t h, cudaStream_t s, int n) {
+  CK(cudaEventRecord(h->ev_fork, s));
+  for (int i = 0; i < n; ++i) CK(cudaStreamWaitEvent(h->streams[i], h->ev_fork, 0));
+  return SPECK_OK;
+}
+speck_status_t join(speck_handle_t h, cudaStream_t s, int n) {
+  for (int i = 0; i < n; ++i) {
+    CK(cudaEventRecord(h->ev_join[i], h->streams[i]));
+    CK(cudaStreamWaitEvent(s, h->ev_join[i], 0));
+  }
+  return SPECK_OK;
+}
+
+BinParams make_bin_params(speck_handle_t h, int pass) {
+  BinParams bp{};
+  bp.pass = pass;
+  bp.use_direct = h->opt_disable_direct ? 0 : 1;
+  for (int c = 0; c < kNumCfg; ++c) {
+    if (pass == 0) bp.cap[c] = sym_map_cap(c);
+    else bp.cap[c] = h->dtype == SPECK_F64 ? num_map_fill<double>(c) : num_map_fill<float>(c);
+  }
+  if (h->opt_force_acc == 2) {  // dense everywhere: every non-trivial row is a single-row block of the largest cfg
+    for (int c = 0; c < kNumCfg - 1; ++c) bp.cap[c] = -1;
+  }
+  return bp;
+}
+
+// Table 2 decision.  need_max / need_avg per row; returns 1 = balance.
+int decide_lb(const LbThresholds& t, int64_t opt, double need_max, double need_sum, int64_t rows, int cfg_of_max,
+              bool forced) {
+  if (forced) return 1;
+  if (opt >= 0) return opt ? 1 : 0;
+  if (rows <= 0 || need_sum <= 0) return 0;
+  const double ratio = need_max / (need_sum / (double)rows);
+  if (cfg_of_max >= t.big_from_cfg) return (ratio > t.ratio_big && rows > t.rows_big) ? 1 : 0;
+  return (ratio > t.ratio && rows > t.rows) ? 1 : 0;
+}
+
+int cfg_for(const BinParams& bp, int64_t need) {
+  for (int c = 0; c < kNumCfg; ++c)
+    if (need <= bp.cap[c]) return c;
+  return kNumCfg;  // does not fit any hash configuration
+}
+
+template <typename V>
+SpgemmArgs<V> base_args(speck_handle_t h, const speck_csr_t* A, const speck_csr_t* B) {
+  SpgemmArgs<V> a{};
+  a.A_rp = A->row_ptr; a.A_col = A->col_idx; a.A_val = static_cast<const V*>(A->values);
+  a.B_rp = B->row_ptr; a.B_col = B->col_idx; a.B_val = static_cast<const V*>(B->values);
+  a.m = A->rows; a.n = B->cols;
+  a.prods = static_cast<const int64_t*>(h->prods.p);
+  a.maxlen = static_cast<const int32_t*>(h->maxlen.p);
+  a.colmin = static_cast<const int32_t*>(h->colmin.p);
+  a.colmax = static_cast<const int32_t*>(h->colmax.p);
+  a.force_acc = (int)h->opt_force_acc;
+  a.dense_window_cap = h->opt_dense_window;
+  a.fixed_g = (int)h->opt_fixed_g;
+  a.cnt = static_cast<int64_t*>(h->cnt.p);
+  a.resume = static_cast<int32_t*>(h->resume.p);
+  a.resume_stride = std::max<int64_t>(h->max_nnza, 1);
+  a.n_dense_rows = reinterpret_cast<unsigned long long*>(static_cast<char*>(h->small.p) + 256);
+  return a;
+}
+
+// Launch one pass (symbolic pass=0 / numeric pass=1) either over the bins (LB on) or over
+// fixed groups of consecutive rows (LB off).
+template <typename V>
+speck_status_t run_pass(speck_handle_t h, int pass, int lb, const int64_t* cat_start, SpgemmArgs<V> a, int64_t need_max,
+                        const BinParams& bp, cudaStream_t s) {
+  const int64_t m = a.m;
+  if (!lb) {
+    // no load balancing: one configuration with room for R rows of the longest size
+    int cfg = -1, R = 1;
+    for (int c = 0; c < kNumCfg; ++c)
+      if (need_max * kMaxGroupRows <= bp.cap[c]) { cfg = c; R = kMaxGroupRows; break; }
+    if (cfg < 0) {
+      cfg = cfg_for(bp, need_max);
+      if (cfg >= kNumCfg) cfg = kNumCfg - 1;
+      R = (int)std::max<int64_t>(1, std::min<int64_t>(kMaxGroupRows, bp.cap[cfg] / std::max<int64_t>(need_max, 1)));
+    }
+    a.rows = nullptr;
+    a.n_entries = m;
+    a.group_rows = R;
+    a.merge = 0;
+    return launch_spgemm<V>(h, cfg, pass, a, s);
+  }
+  const int ns = (int)std::max<int64_t>(1, std::min<int64_t>(h->opt_streams, kMaxStreams));
+  speck_status_t st = fork(h, s, ns);
+  if (st) return st;
+  int si = 0;
+  const int32_t* bins = static_cast<const int32_t*>(h->bins.p);
+  // largest configurations first so long rows start early
+  for (int c = kNumCfg - 1; c >= 0; --c) {
+    const int cat = CAT_CFG0 + c;
+    const int64_t n = cat_start[cat + 1] - cat_start[cat];
+    if (n <= 0) continue;
+    SpgemmArgs<V> b = a;
+    b.rows = bins + cat_start[cat];
+    b.n_entries = n;
+    if (c == 0) {
+      b.group_rows = kMaxGroupRows;
+      b.merge = 1;
+      b.merge_cap = bp.cap[0] + 1;  // merge while the sum stays <= cap (strict < cap+1)
+    } else {
+      b.group_rows = 1;
+      b.merge = 0;
+    }
+    st = launch_spgemm<V>(h, c, pass, b, h->streams[si]);
+    if (st) return st;
+    si = (si + 1) % ns;
+  }
+  if (pass == 1) {
+    const int64_t n = cat_start[CAT_DIRECT + 1] - cat_start[CAT_DIRECT];
+    if (n > 0) {
+      // GD lanes per row: average length of B rows
+      const double avg = h->B_rows > 0 ? (double)h->B_nnz / (double)h->B_rows : 1.0;
+      const int gd = pow2_clamp(avg, 1, 32);
+      const int64_t rows_per_cta = 256 / gd;
+      const unsigned grid = (unsigned)std::min<int64_t>((n + rows_per_cta - 1) / rows_per_cta, (int64_t)h->num_sms * 16);
+      const int32_t* rows = bins + cat_start[CAT_DIRECT];
+      cudaStream_t ds = h->streams[si];
+#define SPECK_DIRECT(GD)                                                                                   \
+  k_direct<V, GD><<<grid, 256, 0, ds>>>(rows, n, a.A_rp, a.A_col, a.A_val, a.B_rp, a.B_col, a.B_val, a.C_rp, \
+                                        a.C_col, a.C_val)
+      switch (gd) {
+        case 1: SPECK_DIRECT(1); break;
+        case 2: SPECK_DIRECT(2); break;
+        case 4: SPECK_DIRECT(4); break;
+        case 8: SPECK_DIRECT(8); break;
+        case 16: SPECK_DIRECT(16); break;
+        default: SPECK_DIRECT(32); break;
+      }
+#undef SPECK_DIRECT
+      CKL();
+    }
+  }
+  return join(h, s, ns);
+}
+
+speck_status_t timing_mark(speck_handle_t h, int i, cudaStream_t s) {
+  if (h->opt_timing) CK(cudaEventRecord(h->ev_t[i], s));
+  return SPECK_OK;
+}
+
+float elapsed(speck_handle_t h, int a, int b) {
+  float ms = 0.f;
+  if (cudaEventElapsedTime(&ms, h->ev_t[a], h->ev_t[b]) != cudaSuccess) {
+    (void)cudaGetLastError();
+    return -1.f;
+  }
+  return ms;
+}
+
+template <typename V>
+speck_status_t analyze_impl(speck_handle_t h, const speck_csr_t* A, const speck_csr_t* B, int64_t* C_rp, int64_t* nnz_c,
+                            cudaStream_t s) {
+  const int64_t m = A->rows;
+  speck_status_t st;
+  h->analyzed = false;
+  h->dtype = A->dtype;
+  h->A_rp = A->row_ptr; h->A_col = A->col_idx; h->A_rows = A->rows; h->A_cols = A->cols; h->A_nnz = A->nnz;
+  h->B_rp = B->row_ptr; h->B_col = B->col_idx; h->B_rows = B->rows; h->B_cols = B->cols; h->B_nnz = B->nnz;
+  std::memset(&h->st, 0, sizeof h->st);
+  if (m == 0) {
+    if (C_rp) CK(cudaMemsetAsync(C_rp, 0, sizeof(int64_t), s));
+    *nnz_c = 0;
+    h->nnz_c = 0;
+    h->analyzed = true;
+    return SPECK_OK;
+  }
+  const int64_t tiles = (m + kBinTile - 1) / kBinTile;
+  if ((st = ensure(h, h->prods, (size_t)m * 8, s))) return st;
+  if ((st = ensure(h, h->maxlen, (size_t)m * 4, s))) return st;
+  if ((st = ensure(h, h->colmin, (size_t)m * 4, s))) return st;
+  if ((st = ensure(h, h->colmax, (size_t)m * 4, s))) return st;
+  if ((st = ensure(h, h->cnt, (size_t)m * 8, s))) return st;
+  if ((st = ensure(h, h->bins, (size_t)m * 4, s))) return st;
+  if ((st = ensure(h, h->hist, (size_t)tiles * CAT_COUNT * 8, s))) return st;
+  if ((st = ensure(h, h->hist_off, ((size_t)tiles * CAT_COUNT + 1) * 8, s))) return st;
+  if ((st = ensure(h, h->small, 4096, s))) return st;
+
+  if (h->opt_validate) {
+    int* bad = reinterpret_cast<int*>(static_cast<char*>(h->small.p) + 512);
+    CK(cudaMemsetAsync(bad, 0, 8, s));
+    k_validate<<<(unsigned)std::min<int64_t>((A->rows + 255) / 256, 4096), 256, 0, s>>>(A->row_ptr, A->col_idx, A->rows, A->cols, bad);
+    k_validate<<<(unsigned)std::min<int64_t>((B->rows + 255) / 256, 4096), 256, 0, s>>>(B->row_ptr, B->col_idx, B->rows, B->cols, bad + 1);
+    CKL();
+    int hb[2];
+    CK(cudaMemcpyAsync(hb, bad, 8, cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    if (hb[0] || hb[1]) return fail(h, SPECK_ERR_INVALID_INPUT, "input CSR %s has unsorted/duplicate/out-of-range columns", hb[0] ? "A" : "B");
+  }
+
+  // ---- 1. row analysis (Alg. 1) ---------------------------------------------------------
+  if ((st = timing_mark(h, 0, s))) return st;
+  AnalysisStats* dstats = static_cast<AnalysisStats*>(h->small.p);
+  CK(cudaMemsetAsync(h->small.p, 0, 4096, s));
+  const int ga = pow2_clamp(m > 0 ? (double)A->nnz / (double)m : 1.0, 1, 32);
+  const unsigned agrid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((m * ga + 255) / 256, (int64_t)h->num_sms * 8));
+  st = launch_analysis(h, ga, [&](auto kern) {
+    kern<<<agrid, 256, 0, s>>>(A->row_ptr, A->col_idx, B->row_ptr, B->col_idx, m, static_cast<int64_t*>(h->prods.p),
+                               static_cast<int32_t*>(h->maxlen.p), static_cast<int32_t*>(h->colmin.p),
+                               static_cast<int32_t*>(h->colmax.p), dstats);
+  });
+  if (st) return st;
+  // symbolic classification histogram per tile (global LB step 1), computed unconditionally
+  const BinParams bps = make_bin_params(h, 0);
+  k_classify<<<(unsigned)tiles, kBinTile, 0, s>>>(A->row_ptr, static_cast<int64_t*>(h->prods.p), nullptr, m, bps,
+                                                 static_cast<int64_t*>(h->hist.p), tiles);
+  CKL();
+  if ((st = launch_scan(h, static_cast<int64_t*>(h->hist.p), tiles * CAT_COUNT, static_cast<int64_t*>(h->hist_off.p),
+                        nullptr, s)))
+    return st;
+  // read back the stats and the bin boundaries (sync #1)
+  {
+    unsigned long long* hp = h->h_pinned;
+    CK(cudaMemcpyAsync(hp, dstats, sizeof(AnalysisStats), cudaMemcpyDeviceToHost, s));
+    for (int c = 0; c <= CAT_COUNT; ++c)
+      CK(cudaMemcpyAsync(hp + 16 + c, static_cast<int64_t*>(h->hist_off.p) + (int64_t)c * tiles, 8,
+                         cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+  }
+  AnalysisStats hs;
+  std::memcpy(&hs, h->h_pinned, sizeof hs);
+  int64_t sym_cat[CAT_COUNT + 1];
+  for (int c = 0; c <= CAT_COUNT; ++c) sym_cat[c] = (int64_t)h->h_pinned[16 + c];
+  h->max_nnza = (int64_t)hs.max_nnza;
+  h->st.products = (int64_t)hs.sum_prods;
+  h->st.max_row_products = (int64_t)hs.max_prods;
+  h->st.rows_direct = (int64_t)hs.n_direct;
+  h->st.rows_empty = (int64_t)hs.n_empty;
+  for (int c = 0; c < CAT_COUNT; ++c) h->st.rows_per_bin_symbolic[c] = sym_cat[c + 1] - sym_cat[c];
+  if ((st = timing_mark(h, 1, s))) return st;
+
+  // resume scratch for multi-window dense rows (largest configuration, one CTA per SM)
+  if ((st = ensure(h, h->resume, (size_t)h->num_sms * (size_t)std::max<int64_t>(h->max_nnza, 1) * 4, s))) return st;
+
+  // ---- 2. symbolic global load balancing decision + binning --------------------------
+  const int cfg_max_sym = cfg_for(bps, (int64_t)hs.max_prods);
+  const int lb_sym = decide_lb(kLbSym, h->opt_lb_sym, (double)hs.max_prods, (double)hs.sum_prods, m, cfg_max_sym,
+                               cfg_max_sym >= kNumCfg - 1 || h->opt_force_acc == 2);
+  h->st.lb_symbolic = lb_sym;
+  SpgemmArgs<V> a = base_args<V>(h, A, B);
+  if (lb_sym) {
+    k_bin_scatter<<<(unsigned)tiles, kBinTile, 0, s>>>(A->row_ptr, static_cast<int64_t*>(h->prods.p), nullptr, m, bps,
+                                                      static_cast<int64_t*>(h->hist_off.p), tiles,
+                                                      static_cast<int32_t*>(h->bins.p), static_cast<int64_t*>(h->cnt.p));
+    CKL();
+  }
+  if ((st = timing_mark(h, 2, s))) return st;
+  // ---- 3. symbolic SpGEMM -------------------------------------------------------------
+  if ((st = run_pass<V>(h, 0, lb_sym, sym_cat, a, (int64_t)hs.max_prods, bps, s))) return st;
+  if ((st = timing_mark(h, 3, s))) return st;
+  // ---- 4. prefix sum -> C row offsets; numeric classification -------------------------
+  unsigned long long* dmax = reinterpret_cast<unsigned long long*>(static_cast<char*>(h->small.p) + 128);
+  if ((st = launch_scan(h, static_cast<int64_t*>(h->cnt.p), m, C_rp, dmax, s))) return st;
+  if ((st = timing_mark(h, 4, s))) return st;
+  const BinParams bpn = make_bin_params(h, 1);
+  k_classify<<<(unsigned)tiles, kBinTile, 0, s>>>(A->row_ptr, static_cast<int64_t*>(h->prods.p), C_rp, m, bpn,
+                                                 static_cast<int64_t*>(h->hist.p), tiles);
+  CKL();
+  if ((st = launch_scan(h, static_cast<int64_t*>(h->hist.p), tiles * CAT_COUNT, static_cast<int64_t*>(h->hist_off.p),
+                        nullptr, s)))
+    return st;
+  {
+    unsigned long long* hp = h->h_pinned;
+    CK(cudaMemcpyAsync(hp, C_rp + m, 8, cudaMemcpyDeviceToHost, s));
+    CK(cudaMemcpyAsync(hp + 1, dmax, 8, cudaMemcpyDeviceToHost, s));
+    for (int c = 0; c <= CAT_COUNT; ++c)
+      CK(cudaMemcpyAsync(hp + 16 + c, static_cast<int64_t*>(h->hist_off.p) + (int64_t)c * tiles, 8,
+                         cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));  // sync #2
+  }
+  h->nnz_c = (int64_t)h->h_pinned[0];
+  h->max_cnt = (int64_t)h->h_pinned[1];
+  for (int c = 0; c <= CAT_COUNT; ++c) h->num_cat_start[c] = (int64_t)h->h_pinned[16 + c];
+  for (int c = 0; c < CAT_COUNT; ++c) h->st.rows_per_bin_numeric[c] = h->num_cat_start[c + 1] - h->num_cat_start[c];
+  *nnz_c = h->nnz_c;
+  h->st.nnz_c = h->nnz_c;
+  if (h->opt_timing) {
+    h->st.ms_analysis = elapsed(h, 0, 1);
+    h->st.ms_symbolic_lb = elapsed(h, 1, 2);
+    h->st.ms_symbolic = elapsed(h, 2, 3);
+    h->st.ms_scan = elapsed(h, 3, 4);
+  }
+  h->analyzed = true;
+  return SPECK_OK;
+}
+
+template <typename V>
+speck_status_t spgemm_impl(speck_handle_t h, const speck_csr_t* A, const speck_csr_t* B, const int64_t* C_rp,
+                           int32_t* C_col, V* C_val, cudaStream_t s) {
+  const int64_t m = A->rows;
+  if (m == 0 || h->nnz_c == 0) return SPECK_OK;
+  speck_status_t st;
+  const int64_t tiles = (m + kBinTile - 1) / kBinTile;
+  const BinParams bpn = make_bin_params(h, 1);
+  const int cfg_max = cfg_for(bpn, h->max_cnt);
+  const int lb = decide_lb(kLbNum, h->opt_lb_num, (double)h->max_cnt, (double)h->nnz_c, m, cfg_max,
+                           cfg_max >= kNumCfg - 1 || h->opt_force_acc == 2);
+  h->st.lb_numeric = lb;
+  h->lb_num = lb;
+  if ((st = timing_mark(h, 5, s))) return st;
+  unsigned long long* ndense = reinterpret_cast<unsigned long long*>(static_cast<char*>(h->small.p) + 256);
+  CK(cudaMemsetAsync(ndense, 0, 8, s));
+  if (lb) {
+    k_bin_scatter<<<(unsigned)tiles, kBinTile, 0, s>>>(A->row_ptr, static_cast<int64_t*>(h->prods.p), C_rp, m, bpn,
+                                                      static_cast<int64_t*>(h->hist_off.p), tiles,
+                                                      static_cast<int32_t*>(h->bins.p), nullptr);
+    CKL();
+  }
+  if ((st = timing_mark(h, 6, s))) return st;
+  SpgemmArgs<V> a = base_args<V>(h, A, B);
+  a.C_rp = C_rp;
+  a.C_col = C_col;
+  a.C_val = C_val;
+  if ((st = run_pass<V>(h, 1, lb, h->num_cat_start, a, h->max_cnt, bpn, s))) return st;
+  if ((st = timing_mark(h, 7, s))) return st;
+  // numeric-stage times and counters are read lazily by speck_get_stats (no sync here)
+  if (h->opt_timing) CK(cudaMemcpyAsync(h->h_pinned + 40, ndense, 8, cudaMemcpyDeviceToHost, s));
+  h->numeric_pending = h->opt_timing != 0;
+  return SPECK_OK;
+}
+
+bool same_problem(speck_handle_t h, const speck_csr_t* A, const speck_csr_t* B) {
+  return h->analyzed && h->A_rp == A->row_ptr && h->A_col == A->col_idx && h->A_rows == A->rows && h->A_cols == A->cols &&
+         h->A_nnz == A->nnz && h->B_rp == B->row_ptr && h->B_col == B->col_idx && h->B_rows == B->rows &&
+         h->B_cols == B->cols && h->B_nnz == B->nnz && h->dtype == A->dtype;
+}
+
+// component kernels -------------------------------------------------------------------
+__global__ void k_block_merge_groups(const int64_t* needs, int64_t n, int64_t cap, uint8_t* flags) {
+  const int64_t g0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) / 32 * 32;
+  if (g0 >= n) return;
+  const int ne = (int)(n - g0 < 32 ? n - g0 : 32);
+  const int l = lane_id();
+  const int64_t need = l < ne ? needs[g0 + l] : 0;
+  const uint32_t st = warp_block_merge(need, ne, cap);
+  if (l < ne) flags[g0 + l] = (st >> l) & 1u;
+}
+
+__global__ void k_group_size(int32_t T, const int64_t* nnzA, const int64_t* prods, const int64_t* maxlen, int64_t n,
+                             int32_t* g) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n) g[i] = local_group_size(T, nnzA[i], prods[i], maxlen[i]);
+}
+
+__global__ void k_hash_probe(const uint32_t* keys, const uint32_t* homes, int64_t n, int32_t size, uint32_t* out_keys,
+                             uint32_t* out_counts) {
+  extern __shared__ uint32_t sm[];
+  uint32_t* sk = sm;
+  uint32_t* sc = sm + size;
+  for (int i = threadIdx.x; i < size; i += blockDim.x) { sk[i] = kEmptyKey; sc[i] = 0; }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    // the pipeline's probe_insert with the home slot injected instead of hash_slot()
+    for (int64_t i = 0; i < n; ++i) {
+      bool is_new;
+      const uint32_t s = probe_insert(sk, (uint32_t)size, homes[i] % (uint32_t)size, keys[i], &is_new);
+      atomicAdd(&sc[s], 1u);
+    }
+  }
+  __syncthreads();
+  for (int i = threadIdx.x; i < size; i += blockDim.x) { out_keys[i] = sk[i]; out_counts[i] = sc[i]; }
+}
+
+}  // namespace
+
+// ======================================================================================
+// C ABI
+// ======================================================================================
+extern "C" {
+
+const char* speck_version(void) { return SPECK_VERSION; }
+
+const char* speck_status_string(speck_status_t s) {
+  switch (s) {
+    case SPECK_OK: return "SPECK_OK";
+    case SPECK_ERR_INVALID_ARGUMENT: return "SPECK_ERR_INVALID_ARGUMENT";
+    case SPECK_ERR_DIMENSION_MISMATCH: return "SPECK_ERR_DIMENSION_MISMATCH";
+    case SPECK_ERR_DTYPE_MISMATCH: return "SPECK_ERR_DTYPE_MISMATCH";
+    case SPECK_ERR_UNSUPPORTED: return "SPECK_ERR_UNSUPPORTED";
+    case SPECK_ERR_OUT_OF_MEMORY: return "SPECK_ERR_OUT_OF_MEMORY";
+    case SPECK_ERR_CUDA: return "SPECK_ERR_CUDA";
+    case SPECK_ERR_NOT_ANALYZED: return "SPECK_ERR_NOT_ANALYZED";
+    case SPECK_ERR_INVALID_INPUT: return "SPECK_ERR_INVALID_INPUT";
+  }
+  return "SPECK_ERR_UNKNOWN";
+}
+
+const char* speck_last_error(speck_handle_t h) { return h ? h->err.c_str() : "null handle"; }
+
+speck_status_t speck_create(speck_handle_t* out, int device) {
+  if (!out) return SPECK_ERR_INVALID_ARGUMENT;
+  *out = nullptr;
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || device < 0 || device >= ndev) {
+    (void)cudaGetLastError();
+    return SPECK_ERR_CUDA;
+  }
+  speck_handle_t h = new (std::nothrow) speck_handle_s();
+  if (!h) return SPECK_ERR_OUT_OF_MEMORY;
+  h->device = device;
+  int prev = 0;
+  cudaGetDevice(&prev);
+  if (cudaSetDevice(device) != cudaSuccess) { delete h; return SPECK_ERR_CUDA; }
+  cudaDeviceGetAttribute(&h->num_sms, cudaDevAttrMultiProcessorCount, device);
+  bool ok = cudaHostAlloc(&h->h_pinned, 64 * 8, cudaHostAllocDefault) == cudaSuccess;
+  for (int i = 0; i < kMaxStreams && ok; ++i) ok = cudaStreamCreateWithFlags(&h->streams[i], cudaStreamNonBlocking) == cudaSuccess;
+  ok = ok && cudaEventCreateWithFlags(&h->ev_fork, cudaEventDisableTiming) == cudaSuccess;
+  for (int i = 0; i < kMaxStreams && ok; ++i) ok = cudaEventCreateWithFlags(&h->ev_join[i], cudaEventDisableTiming) == cudaSuccess;
+  for (int i = 0; i < 8 && ok; ++i) ok = cudaEventCreate(&h->ev_t[i]) == cudaSuccess;
+  if (ok) ok = set_smem_attrs<float>(h) == SPECK_OK && set_smem_attrs<double>(h) == SPECK_OK;
+  cudaSetDevice(prev);
+  if (!ok) {
+    (void)cudaGetLastError();
+    speck_destroy(h);
+    return SPECK_ERR_CUDA;
+  }
+  *out = h;
+  return SPECK_OK;
+}
+
+speck_status_t speck_destroy(speck_handle_t h) {
+  if (!h) return SPECK_ERR_INVALID_ARGUMENT;
+  int prev = 0;
+  cudaGetDevice(&prev);
+  cudaSetDevice(h->device);
+  cudaDeviceSynchronize();
+  Buf* bufs[] = {&h->prods, &h->maxlen, &h->colmin, &h->colmax, &h->cnt, &h->hist, &h->hist_off, &h->bins, &h->stats,
+                 &h->scan_status, &h->resume, &h->small};
+  for (Buf* b : bufs)
+    if (b->p) cudaFree(b->p);
+  if (h->h_pinned) cudaFreeHost(h->h_pinned);
+  for (int i = 0; i < kMaxStreams; ++i) {
+    if (h->streams[i]) cudaStreamDestroy(h->streams[i]);
+    if (h->ev_join[i]) cudaEventDestroy(h->ev_join[i]);
+  }
+  if (h->ev_fork) cudaEventDestroy(h->ev_fork);
+  for (int i = 0; i < 8; ++i)
+    if (h->ev_t[i]) cudaEventDestroy(h->ev_t[i]);
+  (void)cudaGetLastError();
+  cudaSetDevice(prev);
+  delete h;
+  return SPECK_OK;
+}
+
+speck_status_t speck_set_option(speck_handle_t h, int option, int64_t v) {
+  if (!h) return SPECK_ERR_INVALID_ARGUMENT;
+  switch (option) {
+    case SPECK_OPT_GLOBAL_LB_SYMBOLIC: h->opt_lb_sym = v; break;
+    case SPECK_OPT_GLOBAL_LB_NUMERIC: h->opt_lb_num = v; break;
+    case SPECK_OPT_FORCE_ACCUMULATOR:
+      if (v < 0 || v > 2) return fail(h, SPECK_ERR_INVALID_ARGUMENT, "FORCE_ACCUMULATOR must be 0..2");
+      h->opt_force_acc = v; break;
+    case SPECK_OPT_DENSE_WINDOW:
+      if (v < 0) return fail(h, SPECK_ERR_INVALID_ARGUMENT, "DENSE_WINDOW must be >= 0");
+      h->opt_dense_window = v; break;
+    case SPECK_OPT_STAGE_TIMING: h->opt_timing = v; break;
+    case SPECK_OPT_VALIDATE: h->opt_validate = v; break;
+    case SPECK_OPT_DISABLE_DIRECT: h->opt_disable_direct = v; break;
+    case SPECK_OPT_FIXED_GROUP_SIZE:
+      if (v < 0 || v > 1024 || (v & (v - 1))) return fail(h, SPECK_ERR_INVALID_ARGUMENT, "FIXED_GROUP_SIZE must be 0 or a power of two <= 1024");
+      h->opt_fixed_g = v; break;
+    case SPECK_OPT_CONCURRENT_STREAMS:
+      if (v < 1 || v > kMaxStreams) return fail(h, SPECK_ERR_INVALID_ARGUMENT, "CONCURRENT_STREAMS must be 1..8");
+      h->opt_streams = v; break;
+    default: return fail(h, SPECK_ERR_INVALID_ARGUMENT, "unknown option %d", option);
+  }
+  return SPECK_OK;
+}
+
+speck_status_t speck_analyze(speck_handle_t h, const speck_csr_t* A, const speck_csr_t* B, int64_t* C_rp, int64_t* nnz_c,
+                             speck_stream_t stream) {
+  if (!h) return SPECK_ERR_INVALID_ARGUMENT;
+  h->err.clear();
+  speck_status_t st;
+  if ((st = check_csr(h, A, "A", false)) || (st = check_csr(h, B, "B", false))) return st;
+  if (!nnz_c) return fail(h, SPECK_ERR_INVALID_ARGUMENT, "nnz_c is NULL");
+  if (!C_rp) return fail(h, SPECK_ERR_INVALID_ARGUMENT, "C_row_ptr is NULL");
+  if (A->cols != B->rows) return fail(h, SPECK_ERR_DIMENSION_MISMATCH, "A.cols (%lld) != B.rows (%lld)", (long long)A->cols, (long long)B->rows);
+  if (A->dtype != B->dtype) return fail(h, SPECK_ERR_DTYPE_MISMATCH, "A and B value types differ");
+  int prev = 0;
+  cudaGetDevice(&prev);
+  if (cudaSetDevice(h->device) != cudaSuccess) return fail(h, SPECK_ERR_CUDA, "cudaSetDevice failed");
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  st = A->dtype == SPECK_F64 ? analyze_impl<double>(h, A, B, C_rp, nnz_c, s) : analyze_impl<float>(h, A, B, C_rp, nnz_c, s);
+  cudaSetDevice(prev);
+  return st;
+}
+
+speck_status_t speck_spgemm(speck_handle_t h, const speck_csr_t* A, const speck_csr_t* B, const int64_t* C_rp,
+                            int32_t* C_col, void* C_val, speck_stream_t stream) {
+  if (!h) return SPECK_ERR_INVALID_ARGUMENT;
+  h->err.clear();
+  speck_status_t st;
+  if ((st = check_csr(h, A, "A", true)) || (st = check_csr(h, B, "B", true))) return st;
+  if (A->cols != B->rows) return fail(h, SPECK_ERR_DIMENSION_MISMATCH, "A.cols != B.rows");
+  if (A->dtype != B->dtype) return fail(h, SPECK_ERR_DTYPE_MISMATCH, "A and B value types differ");
+  if (!same_problem(h, A, B)) return fail(h, SPECK_ERR_NOT_ANALYZED, "speck_spgemm without a matching speck_analyze");
+  if (h->nnz_c > 0 && (!C_rp || !C_col || !C_val)) return fail(h, SPECK_ERR_INVALID_ARGUMENT, "C arrays are NULL");
+  int prev = 0;
+  cudaGetDevice(&prev);
+  if (cudaSetDevice(h->device) != cudaSuccess) return fail(h, SPECK_ERR_CUDA, "cudaSetDevice failed");
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  st = A->dtype == SPECK_F64 ? spgemm_impl<double>(h, A, B, C_rp, C_col, static_cast<double*>(C_val), s)
+                             : spgemm_impl<float>(h, A, B, C_rp, C_col, static_cast<float*>(C_val), s);
+  cudaSetDevice(prev);
+  return st;
+}
+
+speck_status_t speck_row_analysis(speck_handle_t h, const speck_csr_t* A, const speck_csr_t* B, int64_t* prods,
+                                  int32_t* maxlen, int32_t* colmin, int32_t* colmax, speck_stream_t stream) {
+  if (!h) return SPECK_ERR_INVALID_ARGUMENT;
+  h->err.clear();
+  speck_status_t st;
+  if ((st = check_csr(h, A, "A", false)) || (st = check_csr(h, B, "B", false))) return st;
+  if (A->cols != B->rows) return fail(h, SPECK_ERR_DIMENSION_MISMATCH, "A.cols != B.rows");
+  const int64_t m = A->rows;
+  if (m == 0) return SPECK_OK;
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  int prev = 0;
+  cudaGetDevice(&prev);
+  cudaSetDevice(h->device);
+  int64_t* pr = prods;
+  if (!pr) {
+    if ((st = ensure(h, h->prods, (size_t)m * 8, s))) { cudaSetDevice(prev); return st; }
+    pr = static_cast<int64_t*>(h->prods.p);
+  }
+  const int ga = pow2_clamp((double)A->nnz / (double)m, 1, 32);
+  const unsigned agrid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((m * ga + 255) / 256, (int64_t)h->num_sms * 8));
+  st = launch_analysis(h, ga, [&](auto kern) {
+    kern<<<agrid, 256, 0, s>>>(A->row_ptr, A->col_idx, B->row_ptr, B->col_idx, m, pr, maxlen, colmin, colmax, nullptr);
+  });
+  cudaSetDevice(prev);
+  return st;
+}
+
+speck_status_t speck_get_stats(speck_handle_t h, speck_stats_t* out) {
+  if (!h || !out) return SPECK_ERR_INVALID_ARGUMENT;
+  if (h->numeric_pending) {
+    if (cudaEventSynchronize(h->ev_t[7]) != cudaSuccess) {
+      (void)cudaGetLastError();
+      return fail(h, SPECK_ERR_CUDA, "stage timing event failed");
+    }
+    h->st.ms_numeric_lb = elapsed(h, 5, 6);
+    h->st.ms_numeric = elapsed(h, 6, 7);
+    h->st.rows_dense_numeric = (int64_t)h->h_pinned[40];
+    h->numeric_pending = false;
+  }
+  h->st.workspace_bytes = ws_bytes(h);
+  h->st.kernel_launches = h->launches;
+  *out = h->st;
+  return SPECK_OK;
+}
+
+speck_status_t speck_block_merge(speck_handle_t h, const int64_t* needs, int64_t n, int64_t cap, uint8_t* flags,
+                                 speck_stream_t stream) {
+  if (!h || (n > 0 && (!needs || !flags)) || n < 0) return SPECK_ERR_INVALID_ARGUMENT;
+  if (n == 0) return SPECK_OK;
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  const int64_t groups = (n + 31) / 32;
+  k_block_merge_groups<<<(unsigned)((groups * 32 + 255) / 256), 256, 0, s>>>(needs, n, cap, flags);
+  CKL();
+  return SPECK_OK;
+}
+
+speck_status_t speck_group_size(speck_handle_t h, int32_t T, const int64_t* nnzA, const int64_t* prods, const int64_t* maxlen,
+                                int64_t n, int32_t* g, speck_stream_t stream) {
+  if (!h || n < 0 || T <= 0 || (n > 0 && (!nnzA || !prods || !maxlen || !g))) return SPECK_ERR_INVALID_ARGUMENT;
+  if (n == 0) return SPECK_OK;
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  k_group_size<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(T, nnzA, prods, maxlen, n, g);
+  CKL();
+  return SPECK_OK;
+}
+
+speck_status_t speck_hash_probe(speck_handle_t h, const uint32_t* keys, const uint32_t* homes, int64_t n, int32_t size,
+                                uint32_t* slot_keys, uint32_t* slot_counts, speck_stream_t stream) {
+  if (!h || size <= 0 || size > 8192 || n < 0 || (n > 0 && (!keys || !homes)) || !slot_keys || !slot_counts)
+    return SPECK_ERR_INVALID_ARGUMENT;
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  k_hash_probe<<<1, 128, (size_t)size * 8, s>>>(keys, homes, n, size, slot_keys, slot_counts);
+  CKL();
+  return SPECK_OK;
+}
+
+speck_status_t speck_exclusive_scan(speck_handle_t h, const int64_t* in, int64_t n, int64_t* out, speck_stream_t stream) {
+  if (!h || n < 0 || (n > 0 && !in) || !out) return SPECK_ERR_INVALID_ARGUMENT;
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  return launch_scan(h, in, n, out, nullptr, s);
+}
+
+}  // extern "C"

@@ -1,0 +1,309 @@
+"""CUDA path (libspeck.so through the C ABI) vs the CPU oracle, element by element.
+
+Bar (north_star): row_ptr and col_idx bit-exact; values within |c - r| <= tol·Σ|a·b|
+(tol 1e-5 fp32, 1e-12 fp64); configs whose values are small integers / dyadic rationals
+(C1, C2) must be bit-exact.  Integer stages (analysis, scan, block merge, group size,
+hash probing) are bit-exact against the oracle's functions.
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import workloads as W
+from conftest import golden
+
+pytestmark = pytest.mark.gpu
+
+sp = pytest.importorskip("paper_conf_ppopp_pargerwms20_b200")
+
+
+@pytest.fixture(scope="module")
+def dev():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_ppopp_pargerwms20_b200 import build
+    build.build()
+    return torch.device("cuda", 0)
+
+
+def gpu_spgemm(A, B, **opts):
+    h = sp.Handle(0, **opts)
+    C = h.spgemm(A.to("cuda"), B.to("cuda"))
+    torch.cuda.synchronize()
+    st = h.stats()
+    h.close()
+    return C, st
+
+
+def assert_parity(A, B, C, exact=False, rows=None):
+    """Compare C (device) with the oracle on all rows or on row blocks [(r0, r1), ...]."""
+    tol = oracle.TOL[np.dtype(np.float64 if A.dtype == torch.float64 else np.float32)]
+    rp_all = C.row_ptr.cpu().numpy()
+    assert rp_all[0] == 0 and np.all(np.diff(rp_all) >= 0)
+    blocks = [(0, A.rows)] if rows is None else rows
+    for r0, r1 in blocks:
+        rp, col, val, scale = oracle.spgemm(A, B, r0, r1)
+        s0, s1 = int(rp_all[r0]), int(rp_all[r1])
+        gcol = C.col[s0:s1].cpu().numpy()
+        gval = C.val[s0:s1].cpu().numpy().astype(np.float64)
+        res = oracle.compare(rp_all[r0:r1 + 1], gcol, gval, rp, col, val, scale, tol)
+        assert res["rp_ok"], f"row_ptr mismatch in rows [{r0},{r1})"
+        assert res["col_mismatch"] == 0, f"col mismatch at {res['first_bad']} in rows [{r0},{r1})"
+        assert res["ok"], f"value tolerance violated: {res}"
+        if exact:
+            assert np.array_equal(gval, val), "values must be bit-exact for this config"
+
+
+# ----------------------------------------------------------------------- components
+def test_row_analysis_bit_exact(dev):
+    for A, B in ((W.rmat(12, 16, seed=3), W.rmat(12, 16, seed=4)), (W.poisson2d(64), W.poisson2d(64)),
+                 (W.random_sparse(300, 200, 0.05, seed=5, empty_rows=0.3), W.random_sparse(200, 500, 0.02, seed=6))):
+        h = sp.Handle(0)
+        got = [t.cpu().numpy() for t in h.row_analysis(A.to(dev), B.to(dev))]
+        want = oracle.row_analysis(A, B)
+        for g, w in zip(got, want[:4]):
+            assert np.array_equal(g, w)
+
+
+@pytest.mark.parametrize("n", [0, 1, 7, 2048, 2049, 4096 * 3, 1_000_003])
+def test_scan(dev, n):
+    h = sp.Handle(0)
+    x = torch.randint(0, 1000, (n,), dtype=torch.int64)
+    out = h.exclusive_scan(x.to(dev)).cpu().numpy()
+    ref = np.zeros(n + 1, np.int64)
+    np.cumsum(x.numpy(), out=ref[1:])
+    assert np.array_equal(out, ref)
+
+
+def test_block_merge_fig3_and_random(dev):
+    h = sp.Handle(0)
+    kv, _ = golden("fig3_block_merge.txt")
+    needs = [int(x) for x in kv["needs"].split()]
+    flags = h.block_merge(torch.tensor(needs, device=dev), int(kv["cap"])).cpu().numpy()
+    starts = np.nonzero(flags)[0]
+    sums = [sum(needs[s:e]) for s, e in zip(starts, list(starts[1:]) + [len(needs)])]
+    assert sums == [int(x) for x in kv["final"].split()]
+    rng = np.random.default_rng(0)
+    for _ in range(20):
+        n = int(rng.integers(1, 2000))
+        cap = int(rng.integers(2, 200))
+        nd = rng.integers(0, cap, n)
+        flags = h.block_merge(torch.tensor(nd, device=dev), cap).cpu().numpy()
+        bs, bl = oracle.block_merge(nd, cap)
+        want = np.zeros(n, np.uint8)
+        want[bs] = 1
+        assert np.array_equal(flags, want)
+
+
+def test_group_size_matches_oracle(dev):
+    h = sp.Handle(0)
+    rng = np.random.default_rng(1)
+    n = 5000
+    T = np.array([64, 128, 256, 512, 1024])
+    for t in T:
+        nnzA = rng.integers(1, 3000, n)
+        maxlen = rng.integers(1, 5000, n)
+        prods = np.minimum(maxlen * nnzA, maxlen + rng.integers(0, 100000, n))
+        g = h.group_size(int(t), torch.tensor(nnzA, device=dev), torch.tensor(prods, device=dev),
+                         torch.tensor(maxlen, device=dev)).cpu().numpy()
+        want = np.array([oracle.group_size(int(t), int(a), int(p), int(m)) for a, p, m in zip(nnzA, prods, maxlen)])
+        assert np.array_equal(g, want)
+
+
+def test_hash_probe_fig4_and_random(dev):
+    h = sp.Handle(0)
+    kv, _ = golden("fig4_hash.txt")
+    enc = lambda s: int(s[1]) * 2 + int(s[3])
+    keys, homes = [], []
+    for tok in kv["inserts"].split():
+        name, hh = tok.split(":")
+        keys.append(enc(name)); homes.append(int(hh))
+    size = int(kv["size"])
+    sk, sc = (t.cpu().numpy().astype(np.int64) for t in h.hash_probe(torch.tensor(keys, device=dev),
+                                                                       torch.tensor(homes, device=dev), size))
+    ok, oc = oracle.hash_insert(keys, homes, size)          # empty slot: -1 on both sides
+    assert np.array_equal(sk, ok) and np.array_equal(sc, oc)
+    rng = np.random.default_rng(2)
+    for _ in range(10):
+        size = int(rng.integers(8, 2048))
+        n = int(rng.integers(1, size))
+        keys = rng.integers(0, 50, n)
+        homes = rng.integers(0, size, n)
+        sk, sc = (t.cpu().numpy().astype(np.int64) for t in h.hash_probe(torch.tensor(keys, device=dev),
+                                                                           torch.tensor(homes, device=dev), size))
+        ok, oc = oracle.hash_insert(keys, homes, size)
+        assert np.array_equal(sk, ok) and np.array_equal(sc, oc)
+
+
+# ----------------------------------------------------------------------- SpGEMM configs
+def test_c1_poisson_bit_exact(dev):
+    A = W.poisson2d(64)
+    C, st = gpu_spgemm(A, A)
+    assert C.nnz == 51972 and st["products"] == 100104
+    assert_parity(A, A, C, exact=True)
+
+
+@pytest.mark.parametrize("nf", [16, 32])
+def test_c2_galerkin_small_bit_exact(dev, nf):
+    A, P, R = W.amg27(nf)
+    AP, _ = gpu_spgemm(A, P)
+    assert_parity(A, P, AP, exact=True)
+    APh = W.CSR(AP.rows, AP.cols, AP.row_ptr.cpu(), AP.col.cpu(), AP.val.cpu())
+    Ac, _ = gpu_spgemm(R, APh)
+    assert_parity(R, APh, Ac, exact=True)
+
+
+@pytest.mark.parametrize("cfg", ["c3", "c4", "c5"])
+def test_small_structured_configs(dev, cfg):
+    (label, A, B), = W.config(cfg, small=True)
+    C, st = gpu_spgemm(A, B)
+    assert_parity(A, B, C)
+
+
+PATHS = [
+    dict(),
+    dict(global_lb_symbolic=0, global_lb_numeric=0),
+    dict(global_lb_symbolic=1, global_lb_numeric=1),
+    dict(force_accumulator=1),
+    dict(force_accumulator=2),
+    dict(force_accumulator=2, dense_window=64),
+    dict(force_accumulator=2, dense_window=3),
+    dict(disable_direct=1),
+    dict(fixed_group_size=1),
+    dict(fixed_group_size=32),
+    dict(fixed_group_size=1024),
+    dict(concurrent_streams=1),
+]
+
+
+@pytest.mark.parametrize("opts", PATHS, ids=lambda d: ",".join(f"{k}={v}" for k, v in d.items()) or "auto")
+def test_path_forcing_same_result(dev, opts):
+    """Every accumulator / load-balancing path must give the oracle's result."""
+    A = W.rmat(11, 16, seed=11, dtype=torch.float32)
+    C, st = gpu_spgemm(A, A, **opts)
+    assert_parity(A, A, C)
+    A2 = W.random_sparse(200, 300, 0.03, seed=12, dtype=torch.float64, empty_rows=0.2, zero_frac=0.2)
+    B2 = W.random_sparse(300, 150, 0.05, seed=13, dtype=torch.float64, empty_rows=0.1)
+    C2, _ = gpu_spgemm(A2, B2, **opts)
+    assert_parity(A2, B2, C2)
+
+
+def test_fig5_dense_window_of_three(dev):
+    """Fig. 5: one row, 6 columns, window 3, products at c0,c2,c4,c4,c5 -> c0=1 c2=1 c4=2 c5=1."""
+    kv, _ = golden("fig5_dense.txt")
+    A = W.CSR(1, 3, torch.tensor([0, 3]), torch.tensor([0, 1, 2], dtype=torch.int32), torch.ones(3, dtype=torch.float64))
+    # B rows: {c0, c4}, {c2, c4}, {c5}  -> products c0, c4, c2, c4, c5
+    B = W.CSR(3, 6, torch.tensor([0, 2, 4, 5]), torch.tensor([0, 4, 2, 4, 5], dtype=torch.int32),
+              torch.ones(5, dtype=torch.float64))
+    C, st = gpu_spgemm(A, B, force_accumulator=2, dense_window=int(kv["window"]))
+    got = [f"{c}:{int(v)}" for c, v in zip(C.col.cpu().tolist(), C.val.cpu().tolist())]
+    assert got == [f"{t.split(':')[1]}:{t.split(':')[2]}" for t in kv["out"].split()]
+
+
+def test_edge_cases(dev):
+    f64 = torch.float64
+    # empty A (0 rows), empty product (nnz 0), rows without products, 1x1, rectangular
+    E = W.CSR(0, 5, torch.zeros(1, dtype=torch.int64), torch.zeros(0, dtype=torch.int32), torch.zeros(0, dtype=f64))
+    B = W.random_sparse(5, 7, 0.5, seed=1)
+    C, _ = gpu_spgemm(E, B)
+    assert C.nnz == 0 and C.row_ptr.cpu().tolist() == [0]
+    Z = W.CSR(4, 5, torch.zeros(5, dtype=torch.int64), torch.zeros(0, dtype=torch.int32), torch.zeros(0, dtype=f64))
+    C, _ = gpu_spgemm(Z, B)
+    assert C.nnz == 0 and C.row_ptr.cpu().tolist() == [0] * 5
+    one = W.CSR(1, 1, torch.tensor([0, 1]), torch.tensor([0], dtype=torch.int32), torch.tensor([3.0], dtype=f64))
+    C, _ = gpu_spgemm(one, one)
+    assert C.col.cpu().tolist() == [0] and C.val.cpu().tolist() == [9.0]
+    A = W.random_sparse(1, 4000, 0.9, seed=2)          # one long row
+    Bt = W.random_sparse(4000, 3000, 0.01, seed=3)
+    C, _ = gpu_spgemm(A, Bt)
+    assert_parity(A, Bt, C)
+    A = W.random_sparse(3000, 1, 0.5, seed=4)         # every row single-NZ (direct path)
+    Bw = W.random_sparse(1, 5000, 0.3, seed=5)
+    C, st = gpu_spgemm(A, Bw)
+    # fp64 a·b: the GPU rounds once; the oracle's long-double product is rounded twice, so
+    # only the tolerance (not bit equality) applies to random fp64 values
+    assert_parity(A, Bw, C)
+    assert st["rows_per_bin_numeric"][1] > 0            # the direct bin was used
+
+
+def test_errors(dev):
+    h = sp.Handle(0)
+    A = W.random_sparse(10, 20, 0.2, seed=1).to(dev)
+    B = W.random_sparse(21, 5, 0.2, seed=2).to(dev)
+    with pytest.raises(sp.SpeckError) as e:
+        h.spgemm(A, B)
+    assert e.value.status == 2
+    B32 = W.random_sparse(20, 5, 0.2, seed=2, dtype=torch.float32).to(dev)
+    with pytest.raises(sp.SpeckError) as e:
+        h.spgemm(A, B32)
+    assert e.value.status == 3
+    B = W.random_sparse(20, 5, 0.2, seed=2).to(dev)
+    C = torch.empty(0)
+    h2 = sp.Handle(0)
+    with pytest.raises(sp.SpeckError) as e:   # numeric before analyze
+        h2.numeric(A, B, torch.zeros(11, dtype=torch.int64, device=dev), torch.empty(1, dtype=torch.int32, device=dev),
+                   torch.empty(1, dtype=torch.float64, device=dev))
+    assert e.value.status == 7
+    bad = W.CSR(2, 3, torch.tensor([0, 2, 3]), torch.tensor([2, 1, 0], dtype=torch.int32), torch.ones(3, dtype=torch.float64))
+    h3 = sp.Handle(0, validate=1)
+    with pytest.raises(sp.SpeckError) as e:
+        h3.spgemm(bad.to(dev), W.random_sparse(3, 3, 0.5, seed=3).to(dev))
+    assert e.value.status == 8
+
+
+def test_handle_reuse_and_stats(dev):
+    h = sp.Handle(0, stage_timing=1)
+    for seed in (1, 2, 3):
+        A = W.rmat(10, 8, seed=seed, dtype=torch.float32)
+        C = h.spgemm(A.to(dev), A.to(dev))
+        torch.cuda.synchronize()
+        assert_parity(A, A, C)
+        st = h.stats()
+        prods, *_ , (sp_, pm) = oracle.row_analysis(A, A)
+        assert st["products"] == sp_ and st["max_row_products"] == pm and st["nnz_c"] == C.nnz
+        assert st["ms_symbolic"] >= 0 and st["ms_numeric"] >= 0
+
+
+# ----------------------------------------------------------------------- full sizes
+def sample_blocks(m, prods, seed, n_blocks=6, width=64):
+    rng = np.random.default_rng(seed)
+    starts = list(rng.integers(0, max(m - width, 1), n_blocks))
+    heavy = np.argsort(prods)[-4:]
+    blocks = [(int(s), int(min(s + width, m))) for s in starts] + [(int(r), int(r) + 1) for r in heavy]
+    blocks.append((m - min(width, m), m))   # ragged tail
+    return blocks
+
+
+def test_c2_full_size_bit_exact(dev):
+    """BASELINE config[1] at full size (128^3), both SpGEMMs of the Galerkin chain, every row."""
+    A, P, R = W.amg27(128, device=dev)
+    h = sp.Handle(0)
+    AP = h.spgemm(A, P)
+    Ac = h.spgemm(R, AP)
+    torch.cuda.synchronize()
+    assert AP.nnz == 317 ** 3 and Ac.nnz == 190 ** 3
+    Ah, Ph, Rh = A.to("cpu"), P.to("cpu"), R.to("cpu")
+    assert_parity(Ah, Ph, AP, exact=True)
+    APh = W.CSR(AP.rows, AP.cols, AP.row_ptr.cpu(), AP.col.cpu(), AP.val.cpu())
+    assert_parity(Rh, APh, Ac, exact=True)
+
+
+@pytest.mark.parametrize("cfg", ["c3", "c4", "c5"])
+def test_full_size_sampled(dev, cfg):
+    (label, A, B), = W.config(cfg, device=dev)
+    h = sp.Handle(0)
+    C = h.spgemm(A, B)
+    torch.cuda.synchronize()
+    st = h.stats()
+    prods, _, cmin, cmax = (t.cpu().numpy() for t in h.row_analysis(A, B))
+    rp = C.row_ptr.cpu().numpy()
+    cnt = np.diff(rp)
+    # properties at any size: monotone offsets, nnz(C) bounds, totals
+    assert rp[0] == 0 and np.all(cnt >= 0) and np.all(cnt <= prods)
+    assert int(prods.sum()) == st["products"] and int(rp[-1]) == C.nnz
+    Ah = A.to("cpu")
+    blocks = sample_blocks(A.rows, prods, seed=7)
+    assert_parity(Ah, Ah, C, rows=blocks)
+    del C
+    torch.cuda.empty_cache()
