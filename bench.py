@@ -344,6 +344,8 @@ def run_speck(args):
                        "model_bytes_per_step": int(model_step),
                        "model_GBps": round(model_step / (ms_per_step * 1e-3) / 1e9, 1),
                        "parallelism": f"row-sharded x{world}" if world > 1 else "single GPU",
+                       "stage_ms": {probs[j][0]: {k[3:]: round(statistics.mean(v_), 4) for (jj, k), v_ in stage_ms.items()
+                                                  if jj == j} for j in range(len(probs))},
                        "step_ms": [round(x, 4) for x in step_ms]},
             "roofline": roofline,
             "cpu_baseline": cpu,

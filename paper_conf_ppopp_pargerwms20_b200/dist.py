@@ -81,10 +81,14 @@ def _default_prods(A, B):
     return default_handle(A.row_ptr.device.index).row_analysis(A, B)[0]
 
 
-def broadcast_csr(M, src: int = 0, group=None):
-    """Replicate a CSR matrix from `src` to every rank (NCCL broadcast of row_ptr/col/val)."""
+def broadcast_csr(M, src: int = 0, group=None, device=None):
+    """Replicate a CSR matrix from `src` to every rank (NCCL broadcast of row_ptr/col/val).
+    Non-source ranks pass M=None; `device` defaults to the current CUDA device."""
     rank = dist.get_rank(group)
-    dev = M.row_ptr.device if M is not None else torch.device("cuda", torch.cuda.current_device())
+    if M is not None:
+        dev = M.row_ptr.device
+    else:
+        dev = torch.device(device) if device is not None else torch.device("cuda", torch.cuda.current_device())
     meta = torch.tensor([M.rows, M.cols, M.col.numel(), 1 if M.val.dtype == torch.float64 else 0] if rank == src
                         else [0, 0, 0, 0], dtype=torch.int64, device=dev)
     dist.broadcast(meta, src, group=group)
