@@ -186,7 +186,8 @@ def run_speck(args):
     log(f"[bench] generated {cfg} in {time.time() - t_gen:.1f}s")
     dtype = probs[0][1].dtype
     v = 8 if dtype == torch.float64 else 4
-    handles = [sp.Handle(local_rank, stage_timing=1) for _ in probs]
+    opts = dict(kv.split("=") for kv in args.opt)
+    handles = [sp.Handle(local_rank, stage_timing=1, **{k: int(v) for k, v in opts.items()}) for _ in probs]
     flush = torch.empty(64 * 1024 * 1024, dtype=torch.float32, device=dev)  # 256 MB > 126 MB L2
 
     state = {}
@@ -443,6 +444,7 @@ def main():
     ap.add_argument("--impl", default="speck", choices=["speck", "reference"])
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--opt", action="append", default=[], help="library option name=value (experiments)")
     ap.add_argument("--cpu-budget", type=float, default=20.0, help="seconds of oracle work for the CPU baseline")
     args = ap.parse_args()
     if args.warmup < 3:

@@ -85,7 +85,8 @@ typedef enum {
   SPECK_OPT_VALIDATE = 5,           /* 1: validate input CSR (sorted, unique, in range) [0] */
   SPECK_OPT_DISABLE_DIRECT = 6,     /* 1: route single-NZ rows through the accumulators [0] */
   SPECK_OPT_FIXED_GROUP_SIZE = 7,   /* >0: use this g for every block instead of the local LB [0] */
-  SPECK_OPT_CONCURRENT_STREAMS = 8  /* number of internal streams for concurrent bins, 1..8 [4] */
+  SPECK_OPT_CONCURRENT_STREAMS = 8, /* number of internal streams for concurrent bins, 1..8 [4] */
+  SPECK_OPT_SEGMENTS = 9            /* 1: split rows beyond the largest map into column segments; 0: windowed dense [1] */
 } speck_option_t;
 
 /* Statistics of the last analyze/spgemm pair (speck_get_stats). */
@@ -97,9 +98,10 @@ typedef struct {
   int64_t rows_empty;        /* rows without products */
   int32_t lb_symbolic;       /* 1 if the global load balancer ran for the symbolic step */
   int32_t lb_numeric;        /* 1 if it ran for the numeric step */
-  int64_t rows_per_bin_symbolic[8]; /* [0]=empty [1]=direct [2..6]=configs 0..4 (cfg 4 incl. dense) [7]=dense */
-  int64_t rows_per_bin_numeric[8];
+  int64_t rows_per_bin_symbolic[8]; /* [0]=empty [1]=direct [2..6]=configs 0..4 [7]=unused */
+  int64_t rows_per_bin_numeric[8];  /* [7]=long rows split into column segments */
   int64_t rows_dense_numeric;    /* rows accumulated with the dense accumulator in the numeric step */
+  int64_t segments;              /* column segments the long numeric rows were split into */
   int64_t workspace_bytes;       /* workspace currently held by the handle */
   int64_t kernel_launches;       /* kernels this handle has launched since speck_create (cumulative) */
   float ms_analysis, ms_symbolic_lb, ms_symbolic, ms_scan, ms_numeric_lb, ms_numeric; /* SPECK_OPT_STAGE_TIMING */

@@ -20,7 +20,8 @@ __global__ void __launch_bounds__(256) k_analysis(const int64_t* __restrict__ A_
                                                   const int64_t* __restrict__ B_rp, const int32_t* __restrict__ B_col,
                                                   int64_t m, int64_t* __restrict__ prods, int32_t* __restrict__ maxlen,
                                                   int32_t* __restrict__ colmin, int32_t* __restrict__ colmax,
-                                                  AnalysisStats* st) {
+                                                  AnalysisStats* st, int32_t* __restrict__ long_rows,
+                                                  unsigned int* n_long) {
   const int sub = threadIdx.x % GA;
   constexpr int RPW = 32 / GA;  // rows per warp and iteration
   const int64_t gwarp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -29,8 +30,14 @@ __global__ void __launch_bounds__(256) k_analysis(const int64_t* __restrict__ A_
   // warp-uniform loop so the GA-wide shuffles always see the whole warp
   for (int64_t wrow0 = gwarp * RPW; wrow0 < m; wrow0 += wstride) {
     const int64_t row = wrow0 + lane_id() / GA;
-    const bool valid = row < m;
-    const int64_t a0 = valid ? A_rp[row] : 0, a1 = valid ? A_rp[row + 1] : 0;
+    bool valid = row < m;
+    int64_t a0 = valid ? A_rp[row] : 0, a1 = valid ? A_rp[row + 1] : 0;
+    if (long_rows && a1 - a0 > kAnaLong) {
+      // very long rows of A (e.g. C4's 200k-NZ rows) go to k_analysis_long: one CTA each
+      if (sub == 0) long_rows[atomicAdd(n_long, 1u)] = (int32_t)row;
+      valid = false;
+      a1 = a0;
+    }
     int64_t p = 0;
     int32_t ml = 0, cmin = INT_MAX, cmax = -1;
     for (int64_t q = a0 + sub; q < a1; q += GA) {
@@ -89,6 +96,60 @@ __global__ void __launch_bounds__(256) k_analysis(const int64_t* __restrict__ A_
     atomicAdd(&st->n_direct, d);
     atomicAdd(&st->n_empty, e);
     atomicMax(&st->max_nnza, ma);
+  }
+}
+
+// Rows of A with more than kAnaLong NZ: one CTA per row, block-wide reduction.
+__global__ void __launch_bounds__(256) k_analysis_long(const int64_t* __restrict__ A_rp, const int32_t* __restrict__ A_col,
+                                                       const int64_t* __restrict__ B_rp, const int32_t* __restrict__ B_col,
+                                                       int64_t* __restrict__ prods, int32_t* __restrict__ maxlen,
+                                                       int32_t* __restrict__ colmin, int32_t* __restrict__ colmax,
+                                                       AnalysisStats* st, const int32_t* __restrict__ long_rows,
+                                                       const unsigned int* n_long) {
+  __shared__ int64_t sp[8];
+  __shared__ int32_t sml[8], smn[8], smx[8];
+  const unsigned n = *n_long;
+  for (unsigned i = blockIdx.x; i < n; i += gridDim.x) {
+    const int32_t row = long_rows[i];
+    const int64_t a0 = A_rp[row], a1 = A_rp[row + 1];
+    int64_t p = 0;
+    int32_t ml = 0, cmin = INT_MAX, cmax = -1;
+    for (int64_t q = a0 + threadIdx.x; q < a1; q += blockDim.x) {
+      const int32_t k = A_col[q];
+      const int64_t b0 = B_rp[k], b1 = B_rp[k + 1];
+      const int64_t len = b1 - b0;
+      p += len;
+      ml = max(ml, (int32_t)len);
+      if (len > 0) {
+        cmin = min(cmin, B_col[b0]);
+        cmax = max(cmax, B_col[b1 - 1]);
+      }
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      p += __shfl_xor_sync(0xffffffffu, p, o);
+      ml = max(ml, __shfl_xor_sync(0xffffffffu, ml, o));
+      cmin = min(cmin, __shfl_xor_sync(0xffffffffu, cmin, o));
+      cmax = max(cmax, __shfl_xor_sync(0xffffffffu, cmax, o));
+    }
+    if (lane_id() == 0) { sp[warp_id()] = p; sml[warp_id()] = ml; smn[warp_id()] = cmin; smx[warp_id()] = cmax; }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      for (int w = 1; w < (int)(blockDim.x / 32); ++w) {
+        p += sp[w]; ml = max(ml, sml[w]); cmin = min(cmin, smn[w]); cmax = max(cmax, smx[w]);
+      }
+      prods[row] = p;
+      if (maxlen) maxlen[row] = ml;
+      if (colmin) colmin[row] = cmin;
+      if (colmax) colmax[row] = cmax;
+      if (st) {
+        atomicAdd(&st->sum_prods, (unsigned long long)p);
+        atomicMax(&st->max_prods, (unsigned long long)p);
+        if (p == 0) atomicAdd(&st->n_empty, 1ull);
+        atomicMax(&st->max_nnza, (unsigned long long)(a1 - a0));
+      }
+    }
+    __syncthreads();
   }
 }
 

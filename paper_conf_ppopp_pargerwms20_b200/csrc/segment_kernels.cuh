@@ -1,0 +1,245 @@
+// segment_kernels.cuh — numeric long rows (beyond the largest hash map).
+//
+// The paper processes a row that needs the largest kernel with windowed dense accumulation,
+// one window after the other inside one block.  B200 keeps that
+// for rows whose window overhead is small ("windows" jobs: one CTA, dense windows of 55.6K
+// (fp32) / 27.7K (fp64) columns, resume positions per referenced B row), and splits the
+// others into *column segments*: consecutive 2^s-column chunks grouped so that each
+// segment's exact size (from the per-chunk counts the symbolic pass recorded) fits the
+// largest hash map at <= 66% fill (ordered hash, sorted write-out), or a single chunk that is
+// accumulated densely.  Segments of one row are independent CTAs writing disjoint, known
+// ranges of the row, so a long, wide, sparse row (C5) or one of a few giant rows (C4) is
+// spread over many SMs.
+#pragma once
+
+#include "spgemm_kernels.cuh"
+
+namespace speck {
+
+enum SegMode : int { SEG_HASH = 0, SEG_DENSE = 1, SEG_WINDOWS = 2 };
+
+// Greedy grouping of a row's chunks [c0, c1] (counts cc) into segments; calls emit(lo_chunk,
+// hi_chunk_exclusive, cnt, out_offset_in_row, dense).  `limit` = max entries of a hashed
+// segment; a chunk above it is a dense segment of its own.
+template <typename F>
+__device__ void plan_row_segments(const int32_t* cc, int c0, int c1, int64_t limit, F&& emit) {
+  int cs = c0;
+  int64_t sum = 0, done = 0;
+  for (int c = c0; c <= c1; ++c) {
+    const int64_t x = cc[c];
+    if (x > limit) {
+      if (sum > 0) emit(cs, c, sum, done, false);
+      done += sum;
+      emit(c, c + 1, x, done, true);
+      done += x;
+      sum = 0;
+      cs = c + 1;
+    } else if (sum + x > limit) {
+      emit(cs, c, sum, done, false);
+      done += sum;
+      sum = x;
+      cs = c;
+    } else {
+      sum += x;
+    }
+  }
+  if (sum > 0) emit(cs, c1 + 1, sum, done, false);
+}
+
+struct SegPlanArgs {
+  const int32_t* cand;     // long-row candidates (the symbolic cfg4 bin)
+  int64_t ncand;
+  const int64_t* C_rp;
+  const int64_t* A_rp;
+  const int64_t* prods;
+  const int32_t* colmin;
+  const int32_t* colmax;
+  const int32_t* chunk_cnt;
+  int nchunks;
+  int shift;
+  int64_t limit;           // numeric long-row threshold = entries of a hashed segment
+  int64_t dense_window;    // columns of one dense window of the largest configuration
+  int prefer_parallel;     // few long rows: always split (parallelism across SMs)
+};
+
+// A row is processed as one "windows" job when its windows cost little next to its products:
+// #windows · nnz(A_i) <= products (each window revisits every referenced B row once).
+__device__ __forceinline__ bool use_windows(const SegPlanArgs& a, int32_t row) {
+  if (a.prefer_parallel) return false;
+  const int64_t range = (int64_t)a.colmax[row] - a.colmin[row] + 1;
+  const int64_t nwin = (range + a.dense_window - 1) / a.dense_window;
+  return nwin * (a.A_rp[row + 1] - a.A_rp[row]) <= a.prods[row];
+}
+
+// Pass 1: number of jobs of every long-row candidate (one thread per candidate).
+__global__ void k_seg_count(SegPlanArgs a, int64_t* __restrict__ nseg) {
+  const int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (e >= a.ncand) return;
+  const int32_t row = a.cand[e];
+  const int64_t cnt = a.C_rp[row + 1] - a.C_rp[row];
+  int64_t n = 0;
+  if (cnt > a.limit) {
+    if (use_windows(a, row)) {
+      n = 1;
+    } else {
+      plan_row_segments(a.chunk_cnt + e * a.nchunks, a.colmin[row] >> a.shift, a.colmax[row] >> a.shift, a.limit,
+                        [&](int, int, int64_t, int64_t, bool) { ++n; });
+    }
+  }
+  nseg[e] = n;
+}
+
+// Pass 2: write the job descriptors at the scanned offsets.
+__global__ void k_seg_emit(SegPlanArgs a, const int64_t* __restrict__ seg_off, Seg* __restrict__ segs) {
+  const int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (e >= a.ncand) return;
+  const int32_t row = a.cand[e];
+  const int64_t c0 = a.C_rp[row];
+  const int64_t cnt = a.C_rp[row + 1] - c0;
+  if (cnt <= a.limit) return;
+  const int32_t lo = a.colmin[row], hi = a.colmax[row];
+  int64_t o = seg_off[e];
+  if (use_windows(a, row)) {
+    Seg s;
+    s.row = row; s.col_lo = lo; s.col_hi = hi + 1; s.cnt = (int32_t)(cnt < 0x7fffffff ? cnt : 0x7fffffff); s.out = c0;
+    s.dense = SEG_WINDOWS; s.pad = 0;
+    segs[o] = s;
+    return;
+  }
+  const int shift = a.shift;
+  plan_row_segments(a.chunk_cnt + e * a.nchunks, lo >> shift, hi >> shift, a.limit,
+                    [&](int ca, int cb, int64_t n, int64_t done, bool dense) {
+                      Seg s;
+                      s.row = row;
+                      s.col_lo = max(lo, ca << shift);
+                      s.col_hi = (int32_t)min((int64_t)hi + 1, (int64_t)cb << shift);
+                      s.cnt = (int32_t)n;
+                      s.out = c0 + done;
+                      const int64_t range = (int64_t)s.col_hi - s.col_lo;
+                      // dense when forced by size, or when the segment is dense enough to skip
+                      // hashing and sorting altogether (18% rule)
+                      s.dense = (dense || (range <= a.dense_window && n * 100 > (int64_t)kDensePct * range)) ? SEG_DENSE
+                                                                                                               : SEG_HASH;
+                      s.pad = 0;
+                      segs[o++] = s;
+                    });
+}
+
+// Dense window [wlo, whi) of a row -> flags/values in shared memory -> compacted, sorted
+// output at `out`; returns the entries written.  Block-wide (barriers inside).
+template <typename V, int T, typename Rng>
+__device__ int64_t dense_window_pass(const SpgemmArgs<V>& p, int64_t a0, int alen, uint32_t* bits, V* dvals,
+                                     uint32_t wlo, uint32_t whi, int64_t out, int64_t* part, Rng rng) {
+  constexpr int NW = T / 32;
+  const int tid = threadIdx.x;
+  const uint32_t range = whi - wlo;
+  const int nwords = (int)((range + 31) / 32);
+  for (int i = tid; i < nwords; i += T) bits[i] = 0u;
+  for (uint32_t i = tid; i < range; i += T) dvals[i] = V(0);
+  __syncthreads();
+  expand_row<1, V>(p, a0, alen, warp_id(), NW,
+                   [&](uint32_t col, V v, bool act) { dense_insert<1, V>(bits, dvals, wlo, col, v, act); }, rng);
+  __syncthreads();
+  int64_t done = 0;
+  for (int base = 0; base < nwords; base += T) {
+    const int wi = base + tid;
+    const uint32_t word = wi < nwords ? bits[wi] : 0u;
+    int64_t tot;
+    const int64_t pre = block_excl_scan<T>((int64_t)__popc(word), part, &tot);
+    uint32_t wd = word;
+    int64_t o = out + done + pre;
+    while (wd) {
+      const int b = __ffs(wd) - 1;
+      wd &= wd - 1;
+      const uint32_t ci = (uint32_t)wi * 32 + b;
+      p.C_col[o] = (int32_t)(wlo + ci);
+      p.C_val[o] = dvals[ci];
+      ++o;
+    }
+    done += tot;
+  }
+  __syncthreads();
+  return done;
+}
+
+// One CTA (the largest configuration, 1 CTA/SM) per job.
+template <typename V>
+__global__ void __launch_bounds__(1024, 1) k_segments(SpgemmArgs<V> p, const Seg* __restrict__ segs) {
+  constexpr int CFG = kNumCfg - 1;
+  constexpr int T = kCfgThreads[CFG];
+  constexpr int NW = T / 32;
+  extern __shared__ __align__(16) unsigned char smem[];
+  __shared__ int64_t part[33];
+  __shared__ int s_wrap;
+  const int tid = threadIdx.x;
+  const Seg sg = segs[blockIdx.x];
+  const int64_t a0 = p.A_rp[sg.row];
+  const int alen = (int)(p.A_rp[sg.row + 1] - a0);
+  const uint32_t lo = (uint32_t)sg.col_lo, hi = (uint32_t)sg.col_hi, range = hi - lo;
+
+  if (sg.dense == SEG_HASH) {
+    uint32_t* keys = reinterpret_cast<uint32_t*>(smem);
+    V* vals = reinterpret_cast<V*>(smem + num_val_offset<V>(CFG));
+    const uint32_t S = num_map_cap<V>(CFG);
+    for (uint32_t i = tid; i < S; i += T) { keys[i] = kEmptyKey; vals[i] = V(0); }
+    if (tid == 0) s_wrap = 0;
+    __syncthreads();
+    int wrapped = 0;
+    expand_row<1, V>(
+        p, a0, alen, warp_id(), NW,
+        [&](uint32_t col, V v, bool act) {
+          uint32_t s = 0;
+          if (act) s = probe_insert_mono(keys, S, mono_slot(col, lo, range, S), col, &wrapped);
+          bool leader;
+          const V sum = warp_key_sum(col, v, leader);
+          if (act && leader) atomicAdd(&vals[s], sum);
+        },
+        SegRange{p.B_col, lo, hi});
+    if (wrapped) s_wrap = 1;
+    __syncthreads();
+    if (!s_wrap) {
+      block_write_ordered<T, V>(keys, vals, S, sg.out, p.C_col, p.C_val, part);
+    } else {
+      // compaction + bitonic sort (a probing run wrapped around)
+      int64_t running = 0;
+      for (uint32_t base = 0; base < S; base += T) {
+        const uint32_t s = base + tid;
+        uint32_t kk = kEmptyKey;
+        V vv = V(0);
+        if (s < S) { kk = keys[s]; vv = vals[s]; }
+        const int64_t fl = kk != kEmptyKey;
+        int64_t tot;
+        const int64_t pos = block_excl_scan<T>(fl, part, &tot);
+        if (fl) { keys[running + pos] = kk; vals[running + pos] = vv; }
+        running += tot;
+        __syncthreads();
+      }
+      smem_bitonic_sort<T, V>(keys, vals, (int)running);
+      for (int i = tid; i < (int)running; i += T) {
+        p.C_col[sg.out + i] = (int32_t)keys[i];
+        p.C_val[sg.out + i] = vals[i];
+      }
+    }
+  } else {
+    const int64_t W = num_dense_window<V>(CFG);
+    uint32_t* bits = reinterpret_cast<uint32_t*>(smem);
+    V* dvals = reinterpret_cast<V*>(smem + ((((W + 31) / 32) * 4 + 15) / 16) * 16);
+    if (sg.dense == SEG_DENSE) {
+      dense_window_pass<V, T>(p, a0, alen, bits, dvals, lo, hi, sg.out, part, SegRange{p.B_col, lo, hi});
+    } else {
+      // whole row, windows in ascending column order with resume positions
+      int32_t* res = p.resume + (int64_t)smid() * p.resume_stride;   // 1 CTA per SM: private slot
+      int32_t* res_next = res + p.resume_stride / 2;
+      for (int f = tid; f < alen; f += T) res[f] = 0;
+      int64_t out = sg.out;
+      for (uint32_t wlo = lo; wlo < hi; wlo = (uint32_t)min((int64_t)hi, (int64_t)wlo + W)) {
+        const uint32_t whi = (uint32_t)min((int64_t)hi, (int64_t)wlo + W);
+        out += dense_window_pass<V, T>(p, a0, alen, bits, dvals, wlo, whi, out, part,
+                                       WindowRange{res, res_next, p.B_col, whi});
+        int32_t* t_ = res; res = res_next; res_next = t_;   // dense_window_pass ends with a barrier
+      }
+    }
+  }
+}
+
+}  // namespace speck

@@ -15,6 +15,7 @@
 
 #include "plan_kernels.cuh"
 #include "spgemm_kernels.cuh"
+#include "segment_kernels.cuh"
 
 #define SPECK_VERSION "speck-b200 0.1.0 (sm_100a)"
 
@@ -42,7 +43,7 @@ struct speck_handle_s {
   int64_t opt_lb_sym = -1, opt_lb_num = -1, opt_force_acc = 0, opt_dense_window = 0, opt_timing = 0, opt_validate = 0,
           opt_disable_direct = 0, opt_fixed_g = 0, opt_streams = 4;
   // workspace
-  Buf prods, maxlen, colmin, colmax, cnt, hist, hist_off, bins, stats, scan_status, resume, small;
+  Buf prods, maxlen, colmin, colmax, cnt, hist, hist_off, bins, stats, scan_status, resume, small, ana_long;
   unsigned long long* h_pinned = nullptr;  // pinned readback area (64 x u64)
   cudaStream_t streams[kMaxStreams] = {};
   cudaEvent_t ev_fork = nullptr, ev_join[kMaxStreams] = {};
@@ -58,6 +59,12 @@ struct speck_handle_s {
   int lb_num = 0;
   bool numeric_pending = false;
   int64_t launches = 0;  // kernels launched by this handle (cumulative)
+  // long-row segments
+  int64_t opt_segments = 1;
+  bool seg_enabled = false;
+  int seg_shift = 15, nchunks = 0;
+  int64_t long_thr = INT64_MAX, n_cand = 0, n_segs = 0, cand_start = 0;
+  Buf chunk_cnt, cand, nseg, seg_off, segs;
 };
 
 namespace {
@@ -109,7 +116,8 @@ speck_status_t ensure(speck_handle_t h, Buf& b, size_t bytes, cudaStream_t s) {
 
 int64_t ws_bytes(speck_handle_t h) {
   return (int64_t)(h->prods.cap + h->maxlen.cap + h->colmin.cap + h->colmax.cap + h->cnt.cap + h->hist.cap +
-                   h->hist_off.cap + h->bins.cap + h->stats.cap + h->scan_status.cap + h->resume.cap + h->small.cap);
+                   h->hist_off.cap + h->bins.cap + h->stats.cap + h->scan_status.cap + h->resume.cap + h->small.cap +
+                   h->ana_long.cap + h->chunk_cnt.cap + h->cand.cap + h->nseg.cap + h->seg_off.cap + h->segs.cap);
 }
 
 speck_status_t check_csr(speck_handle_t h, const speck_csr_t* M, const char* name, bool need_values) {
@@ -124,24 +132,42 @@ speck_status_t check_csr(speck_handle_t h, const speck_csr_t* M, const char* nam
   return SPECK_OK;
 }
 
-template <typename F>
-speck_status_t launch_analysis(speck_handle_t h, int ga, F&& f) {
-  switch (ga) {
-    case 1: f(k_analysis<1>); break;
-    case 2: f(k_analysis<2>); break;
-    case 4: f(k_analysis<4>); break;
-    case 8: f(k_analysis<8>); break;
-    case 16: f(k_analysis<16>); break;
-    default: f(k_analysis<32>); break;
-  }
-  CKL();
-  return SPECK_OK;
-}
-
 int pow2_clamp(double x, int lo, int hi) {
   int p = lo;
   while (p * 2 <= hi && (double)(p * 2) <= x) p *= 2;
   return p;
+}
+
+// Row analysis (Alg. 1): GA lanes per row (GA ~ average row length of A), rows longer than
+// kAnaLong deferred to one CTA each.  `st` may be null (no statistics).
+speck_status_t run_analysis(speck_handle_t h, const speck_csr_t* A, const speck_csr_t* B, int64_t* prods,
+                            int32_t* maxlen, int32_t* colmin, int32_t* colmax, AnalysisStats* st, cudaStream_t s) {
+  const int64_t m = A->rows;
+  speck_status_t r;
+  if ((r = ensure(h, h->ana_long, (size_t)(A->nnz / kAnaLong + 1) * 4, s))) return r;
+  if ((r = ensure(h, h->small, 4096, s))) return r;
+  unsigned* nlong = reinterpret_cast<unsigned*>(static_cast<char*>(h->small.p) + 640);
+  int32_t* lrows = static_cast<int32_t*>(h->ana_long.p);
+  CK(cudaMemsetAsync(nlong, 0, 4, s));
+  const int ga = pow2_clamp(m > 0 ? (double)A->nnz / (double)m : 1.0, 1, 32);
+  const unsigned agrid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((m * ga + 255) / 256, (int64_t)h->num_sms * 8));
+#define SPECK_ANA(GA)                                                                                        \
+  k_analysis<GA><<<agrid, 256, 0, s>>>(A->row_ptr, A->col_idx, B->row_ptr, B->col_idx, m, prods, maxlen, colmin, \
+                                       colmax, st, lrows, nlong)
+  switch (ga) {
+    case 1: SPECK_ANA(1); break;
+    case 2: SPECK_ANA(2); break;
+    case 4: SPECK_ANA(4); break;
+    case 8: SPECK_ANA(8); break;
+    case 16: SPECK_ANA(16); break;
+    default: SPECK_ANA(32); break;
+  }
+#undef SPECK_ANA
+  CKL();
+  k_analysis_long<<<(unsigned)h->num_sms * 2, 256, 0, s>>>(A->row_ptr, A->col_idx, B->row_ptr, B->col_idx, prods, maxlen,
+                                                           colmin, colmax, st, lrows, nlong);
+  CKL();
+  return SPECK_OK;
 }
 
 // kernel function pointer for (cfg, pass, V)
@@ -177,6 +203,7 @@ speck_status_t set_smem_attrs(speck_handle_t h) {
   for (int c = 0; c < kNumCfg; ++c)
     for (int pass = 0; pass < 2; ++pass)
       CK(cudaFuncSetAttribute(spgemm_fn<V>(c, pass), cudaFuncAttributeMaxDynamicSharedMemorySize, kCfgMapBytes[c]));
+  CK(cudaFuncSetAttribute(k_segments<V>, cudaFuncAttributeMaxDynamicSharedMemorySize, kCfgMapBytes[kNumCfg - 1]));
   return SPECK_OK;
 }
 
@@ -211,14 +238,34 @@ BinParams make_bin_params(speck_handle_t h, int pass) {
   BinParams bp{};
   bp.pass = pass;
   bp.use_direct = h->opt_disable_direct ? 0 : 1;
+  bp.long_thr = INT64_MAX;
   for (int c = 0; c < kNumCfg; ++c) {
-    if (pass == 0) bp.cap[c] = sym_map_cap(c);
+    if (pass == 0) bp.cap[c] = sym_map_fill(c);
     else bp.cap[c] = h->dtype == SPECK_F64 ? num_map_fill<double>(c) : num_map_fill<float>(c);
+  }
+  if (h->seg_enabled) {
+    // every row that may exceed the largest numeric map is a symbolic cfg4 row, so that the
+    // symbolic pass records its per-chunk counts; such rows become numeric segments
+    if (pass == 0) bp.cap[kNumCfg - 2] = std::min<int64_t>(bp.cap[kNumCfg - 2], h->long_thr);
+    else bp.long_thr = h->long_thr;
   }
   if (h->opt_force_acc == 2) {  // dense everywhere: every non-trivial row is a single-row block of the largest cfg
     for (int c = 0; c < kNumCfg - 1; ++c) bp.cap[c] = -1;
   }
   return bp;
+}
+
+// Segment geometry for long numeric rows (segment_kernels.cuh); decided before the analysis.
+template <typename V>
+void plan_segments(speck_handle_t h, int64_t ncols) {
+  h->long_thr = num_map_fill<V>(kNumCfg - 1);
+  int s = 0;
+  while ((int64_t)1 << (s + 1) <= num_dense_window<V>(kNumCfg - 1)) ++s;
+  h->seg_shift = s;
+  h->nchunks = (int)((ncols + ((int64_t)1 << s) - 1) >> s);
+  h->seg_enabled = h->opt_force_acc != 2 && h->opt_segments != 0 && h->nchunks >= 1 && h->nchunks <= kMaxChunks;
+  h->n_cand = 0;
+  h->n_segs = 0;
 }
 
 // Table 2 decision.  need_max / need_avg per row; returns 1 = balance.
@@ -253,9 +300,29 @@ SpgemmArgs<V> base_args(speck_handle_t h, const speck_csr_t* A, const speck_csr_
   a.fixed_g = (int)h->opt_fixed_g;
   a.cnt = static_cast<int64_t*>(h->cnt.p);
   a.resume = static_cast<int32_t*>(h->resume.p);
-  a.resume_stride = std::max<int64_t>(h->max_nnza, 1);
+  a.resume_stride = 2 * std::max<int64_t>(h->max_nnza, 1);   // two buffers (cur / next) per SM slot
   a.n_dense_rows = reinterpret_cast<unsigned long long*>(static_cast<char*>(h->small.p) + 256);
   return a;
+}
+
+template <typename V>
+SegPlanArgs seg_plan_args(speck_handle_t h, const int64_t* C_rp) {
+  SegPlanArgs s{};
+  s.cand = static_cast<const int32_t*>(h->cand.p);
+  s.ncand = h->n_cand;
+  s.C_rp = C_rp;
+  s.A_rp = h->A_rp;
+  s.prods = static_cast<const int64_t*>(h->prods.p);
+  s.colmin = static_cast<const int32_t*>(h->colmin.p);
+  s.colmax = static_cast<const int32_t*>(h->colmax.p);
+  s.chunk_cnt = static_cast<const int32_t*>(h->chunk_cnt.p);
+  s.nchunks = h->nchunks;
+  s.shift = h->seg_shift;
+  s.limit = h->long_thr;
+  s.dense_window = num_dense_window<V>(kNumCfg - 1);
+  // few candidates: split every long row so its work spreads over the SMs
+  s.prefer_parallel = h->n_cand < 4 * (int64_t)h->num_sms ? 1 : 0;
+  return s;
 }
 
 // Launch one pass (symbolic pass=0 / numeric pass=1) either over the bins (LB on) or over
@@ -281,10 +348,26 @@ speck_status_t run_pass(speck_handle_t h, int pass, int lb, const int64_t* cat_s
     return launch_spgemm<V>(h, cfg, pass, a, s);
   }
   const int ns = (int)std::max<int64_t>(1, std::min<int64_t>(h->opt_streams, kMaxStreams));
-  speck_status_t st = fork(h, s, ns);
-  if (st) return st;
+  speck_status_t st;
+  const bool segs = pass == 1 && h->seg_enabled && h->n_segs > 0;
+  if (segs) {
+    // segment descriptors of the long rows (offsets were scanned during analyze)
+    if ((st = ensure(h, h->segs, (size_t)h->n_segs * sizeof(Seg), s))) return st;
+    const int64_t nc = h->n_cand;
+    k_seg_emit<<<(unsigned)((nc + 127) / 128), 128, 0, s>>>(seg_plan_args<V>(h, a.C_rp),
+                                                           static_cast<const int64_t*>(h->seg_off.p),
+                                                           static_cast<Seg*>(h->segs.p));
+    CKL();
+  }
+  if ((st = fork(h, s, ns))) return st;
   int si = 0;
   const int32_t* bins = static_cast<const int32_t*>(h->bins.p);
+  if (segs) {
+    k_segments<V><<<(unsigned)h->n_segs, kCfgThreads[kNumCfg - 1], kCfgMapBytes[kNumCfg - 1], h->streams[si]>>>(
+        a, static_cast<const Seg*>(h->segs.p));
+    CKL();
+    si = (si + 1) % ns;
+  }
   // largest configurations first so long rows start early
   for (int c = kNumCfg - 1; c >= 0; --c) {
     const int cat = CAT_CFG0 + c;
@@ -300,6 +383,12 @@ speck_status_t run_pass(speck_handle_t h, int pass, int lb, const int64_t* cat_s
     } else {
       b.group_rows = 1;
       b.merge = 0;
+    }
+    if (pass == 0 && c == kNumCfg - 1 && h->seg_enabled && h->n_cand > 0) {
+      b.chunk_cnt = static_cast<int32_t*>(h->chunk_cnt.p);   // entry e of this bin -> chunk_cnt[e]
+      b.nchunks = h->nchunks;
+      b.chunk_shift = h->seg_shift;
+      b.long_thr = h->long_thr;
     }
     st = launch_spgemm<V>(h, c, pass, b, h->streams[si]);
     if (st) return st;
@@ -357,6 +446,7 @@ speck_status_t analyze_impl(speck_handle_t h, const speck_csr_t* A, const speck_
   h->A_rp = A->row_ptr; h->A_col = A->col_idx; h->A_rows = A->rows; h->A_cols = A->cols; h->A_nnz = A->nnz;
   h->B_rp = B->row_ptr; h->B_col = B->col_idx; h->B_rows = B->rows; h->B_cols = B->cols; h->B_nnz = B->nnz;
   std::memset(&h->st, 0, sizeof h->st);
+  plan_segments<V>(h, B->cols);
   if (m == 0) {
     if (C_rp) CK(cudaMemsetAsync(C_rp, 0, sizeof(int64_t), s));
     *nnz_c = 0;
@@ -391,14 +481,9 @@ speck_status_t analyze_impl(speck_handle_t h, const speck_csr_t* A, const speck_
   if ((st = timing_mark(h, 0, s))) return st;
   AnalysisStats* dstats = static_cast<AnalysisStats*>(h->small.p);
   CK(cudaMemsetAsync(h->small.p, 0, 4096, s));
-  const int ga = pow2_clamp(m > 0 ? (double)A->nnz / (double)m : 1.0, 1, 32);
-  const unsigned agrid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((m * ga + 255) / 256, (int64_t)h->num_sms * 8));
-  st = launch_analysis(h, ga, [&](auto kern) {
-    kern<<<agrid, 256, 0, s>>>(A->row_ptr, A->col_idx, B->row_ptr, B->col_idx, m, static_cast<int64_t*>(h->prods.p),
-                               static_cast<int32_t*>(h->maxlen.p), static_cast<int32_t*>(h->colmin.p),
-                               static_cast<int32_t*>(h->colmax.p), dstats);
-  });
-  if (st) return st;
+  if ((st = run_analysis(h, A, B, static_cast<int64_t*>(h->prods.p), static_cast<int32_t*>(h->maxlen.p),
+                         static_cast<int32_t*>(h->colmin.p), static_cast<int32_t*>(h->colmax.p), dstats, s)))
+    return st;
   // symbolic classification histogram per tile (global LB step 1), computed unconditionally
   const BinParams bps = make_bin_params(h, 0);
   k_classify<<<(unsigned)tiles, kBinTile, 0, s>>>(A->row_ptr, static_cast<int64_t*>(h->prods.p), nullptr, m, bps,
@@ -429,13 +514,26 @@ speck_status_t analyze_impl(speck_handle_t h, const speck_csr_t* A, const speck_
   if ((st = timing_mark(h, 1, s))) return st;
 
   // resume scratch for multi-window dense rows (largest configuration, one CTA per SM)
-  if ((st = ensure(h, h->resume, (size_t)h->num_sms * (size_t)std::max<int64_t>(h->max_nnza, 1) * 4, s))) return st;
+  if ((st = ensure(h, h->resume, (size_t)h->num_sms * 2 * (size_t)std::max<int64_t>(h->max_nnza, 1) * 4, s))) return st;
 
   // ---- 2. symbolic global load balancing decision + binning --------------------------
   const int cfg_max_sym = cfg_for(bps, (int64_t)hs.max_prods);
   const int lb_sym = decide_lb(kLbSym, h->opt_lb_sym, (double)hs.max_prods, (double)hs.sum_prods, m, cfg_max_sym,
                                cfg_max_sym >= kNumCfg - 1 || h->opt_force_acc == 2);
   h->st.lb_symbolic = lb_sym;
+  if (h->seg_enabled && lb_sym) {
+    // long-row candidates = the symbolic bin of the largest configuration
+    h->cand_start = sym_cat[CAT_CFG0 + kNumCfg - 1];
+    h->n_cand = sym_cat[CAT_CFG0 + kNumCfg] - h->cand_start;
+    const size_t bytes = (size_t)h->n_cand * (size_t)h->nchunks * 4;
+    if (h->n_cand > 0 && (bytes > ((size_t)4 << 30) || ensure(h, h->chunk_cnt, bytes, s) != SPECK_OK)) {
+      (void)cudaGetLastError();
+      h->seg_enabled = false;   // too many candidates for the chunk table: dense windows instead
+      h->n_cand = 0;
+    }
+  } else {
+    h->n_cand = 0;
+  }
   SpgemmArgs<V> a = base_args<V>(h, A, B);
   if (lb_sym) {
     k_bin_scatter<<<(unsigned)tiles, kBinTile, 0, s>>>(A->row_ptr, static_cast<int64_t*>(h->prods.p), nullptr, m, bps,
@@ -458,10 +556,27 @@ speck_status_t analyze_impl(speck_handle_t h, const speck_csr_t* A, const speck_
   if ((st = launch_scan(h, static_cast<int64_t*>(h->hist.p), tiles * CAT_COUNT, static_cast<int64_t*>(h->hist_off.p),
                         nullptr, s)))
     return st;
+  // numeric long rows: segments per candidate (exact sizes from the symbolic chunk counts)
+  if (h->seg_enabled && h->n_cand > 0) {
+    const int64_t nc = h->n_cand;
+    if ((st = ensure(h, h->cand, (size_t)nc * 4, s))) return st;
+    if ((st = ensure(h, h->nseg, (size_t)nc * 8, s))) return st;
+    if ((st = ensure(h, h->seg_off, (size_t)(nc + 1) * 8, s))) return st;
+    CK(cudaMemcpyAsync(h->cand.p, static_cast<int32_t*>(h->bins.p) + h->cand_start, (size_t)nc * 4,
+                       cudaMemcpyDeviceToDevice, s));
+    k_seg_count<<<(unsigned)((nc + 127) / 128), 128, 0, s>>>(seg_plan_args<V>(h, C_rp),
+                                                            static_cast<int64_t*>(h->nseg.p));
+    CKL();
+    if ((st = launch_scan(h, static_cast<int64_t*>(h->nseg.p), nc, static_cast<int64_t*>(h->seg_off.p), nullptr, s)))
+      return st;
+  }
   {
     unsigned long long* hp = h->h_pinned;
     CK(cudaMemcpyAsync(hp, C_rp + m, 8, cudaMemcpyDeviceToHost, s));
     CK(cudaMemcpyAsync(hp + 1, dmax, 8, cudaMemcpyDeviceToHost, s));
+    hp[2] = 0;
+    if (h->seg_enabled && h->n_cand > 0)
+      CK(cudaMemcpyAsync(hp + 2, static_cast<int64_t*>(h->seg_off.p) + h->n_cand, 8, cudaMemcpyDeviceToHost, s));
     for (int c = 0; c <= CAT_COUNT; ++c)
       CK(cudaMemcpyAsync(hp + 16 + c, static_cast<int64_t*>(h->hist_off.p) + (int64_t)c * tiles, 8,
                          cudaMemcpyDeviceToHost, s));
@@ -469,6 +584,8 @@ speck_status_t analyze_impl(speck_handle_t h, const speck_csr_t* A, const speck_
   }
   h->nnz_c = (int64_t)h->h_pinned[0];
   h->max_cnt = (int64_t)h->h_pinned[1];
+  h->n_segs = (int64_t)h->h_pinned[2];
+  h->st.segments = h->n_segs;
   for (int c = 0; c <= CAT_COUNT; ++c) h->num_cat_start[c] = (int64_t)h->h_pinned[16 + c];
   for (int c = 0; c < CAT_COUNT; ++c) h->st.rows_per_bin_numeric[c] = h->num_cat_start[c + 1] - h->num_cat_start[c];
   *nnz_c = h->nnz_c;
@@ -624,7 +741,8 @@ speck_status_t speck_destroy(speck_handle_t h) {
   cudaSetDevice(h->device);
   cudaDeviceSynchronize();
   Buf* bufs[] = {&h->prods, &h->maxlen, &h->colmin, &h->colmax, &h->cnt, &h->hist, &h->hist_off, &h->bins, &h->stats,
-                 &h->scan_status, &h->resume, &h->small};
+                 &h->scan_status, &h->resume, &h->small, &h->ana_long, &h->chunk_cnt, &h->cand, &h->nseg,
+                 &h->seg_off, &h->segs};
   for (Buf* b : bufs)
     if (b->p) cudaFree(b->p);
   if (h->h_pinned) cudaFreeHost(h->h_pinned);
@@ -661,6 +779,7 @@ speck_status_t speck_set_option(speck_handle_t h, int option, int64_t v) {
     case SPECK_OPT_CONCURRENT_STREAMS:
       if (v < 1 || v > kMaxStreams) return fail(h, SPECK_ERR_INVALID_ARGUMENT, "CONCURRENT_STREAMS must be 1..8");
       h->opt_streams = v; break;
+    case SPECK_OPT_SEGMENTS: h->opt_segments = v; break;
     default: return fail(h, SPECK_ERR_INVALID_ARGUMENT, "unknown option %d", option);
   }
   return SPECK_OK;
@@ -723,11 +842,7 @@ speck_status_t speck_row_analysis(speck_handle_t h, const speck_csr_t* A, const 
     if ((st = ensure(h, h->prods, (size_t)m * 8, s))) { cudaSetDevice(prev); return st; }
     pr = static_cast<int64_t*>(h->prods.p);
   }
-  const int ga = pow2_clamp((double)A->nnz / (double)m, 1, 32);
-  const unsigned agrid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((m * ga + 255) / 256, (int64_t)h->num_sms * 8));
-  st = launch_analysis(h, ga, [&](auto kern) {
-    kern<<<agrid, 256, 0, s>>>(A->row_ptr, A->col_idx, B->row_ptr, B->col_idx, m, pr, maxlen, colmin, colmax, nullptr);
-  });
+  st = run_analysis(h, A, B, pr, maxlen, colmin, colmax, nullptr, s);
   cudaSetDevice(prev);
   return st;
 }

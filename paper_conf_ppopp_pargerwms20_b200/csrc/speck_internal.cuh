@@ -23,21 +23,41 @@ namespace speck {
 constexpr int kNumCfg = 5;
 constexpr int kCfgThreads[kNumCfg] = {64, 128, 256, 512, 1024};
 // accumulator (hash map / dense window) bytes per configuration
-constexpr int kCfgMapBytes[kNumCfg] = {11776, 26112, 54272, 111616, 225280};
+constexpr int kCfgMapBytes[kNumCfg] = {11264, 25856, 54272, 111616, 225280};
 __host__ __device__ constexpr int cfg_map_bytes(int c) {
-  return c == 0 ? 11776 : c == 1 ? 26112 : c == 2 ? 54272 : c == 3 ? 111616 : 225280;
+  return c == 0 ? 11264 : c == 1 ? 25856 : c == 2 ? 54272 : c == 3 ? 111616 : 225280;
 }
+// B200: 228 KB shared memory per SM (233472 B), 1 KB reserved per resident CTA, <= 227 KB per CTA
+constexpr int kSmemPerSM = 233472;
+constexpr int kSmemPerCtaMax = 232448;
 static_assert(cfg_map_bytes(4) == kCfgMapBytes[4] && cfg_map_bytes(0) == kCfgMapBytes[0], "ladder");
 constexpr int kMaxGroupRows = 32;     // rows per block (5-bit local row id)
 constexpr int kBinTile = 1024;        // rows per binning tile
 constexpr int kMaxStreams = 8;
+constexpr int64_t kAnaLong = 4096;    // rows of A longer than this get a whole CTA in the analysis
 
 // categories (bins) of a row for one pass
 enum Cat : int {
   CAT_EMPTY = 0,  // no products: row of C is empty
   CAT_DIRECT = 1, // single NZ in the row of A
   CAT_CFG0 = 2,   // CAT_CFG0 + j = configuration j (cfg0 bin = merged small rows)
-  CAT_COUNT = CAT_CFG0 + kNumCfg
+  CAT_LONG = CAT_CFG0 + kNumCfg,  // numeric rows beyond the largest map: split into column segments
+  CAT_COUNT = CAT_LONG + 1
+};
+
+// Long rows (numeric nnz beyond the largest hash map) are split into column segments whose
+// exact sizes come from per-chunk counts recorded by the symbolic pass: chunks of 2^s
+// columns (2^s <= one dense window of the largest configuration: s = 15 fp32, 14 fp64), at
+// most kMaxChunks per row.
+constexpr int kMaxChunks = 1024;
+struct Seg {
+  int32_t row;
+  int32_t col_lo;   // first column of the segment
+  int32_t col_hi;   // one past the last column
+  int32_t cnt;      // exact entries of C in [col_lo, col_hi)
+  int64_t out;      // position of the segment's first entry in C
+  int32_t dense;    // 1: dense window accumulator, 0: ordered hash map
+  int32_t pad;
 };
 
 constexpr uint32_t kEmptyKey = 0xFFFFFFFFu;
@@ -53,6 +73,11 @@ __host__ __device__ constexpr int num_slot_bytes() { return 4 + (int)sizeof(V); 
 
 // capacity (slots) of a configuration's hash map
 __host__ __device__ inline uint32_t sym_map_cap(int cfg) { return (uint32_t)(cfg_map_bytes(cfg) / 4); }
+// Symbolic rows are binned by products, an upper bound of their distinct columns.
+// The paper relies on the average compaction of ~7 to keep the map sparse; for
+// inputs without compaction (R-MAT C5: ~1.05) the bound is tight, so B200 bins against 66% of
+// the slots as in the numeric step — linear probing stays short either way.
+__host__ __device__ inline uint32_t sym_map_fill(int cfg) { return (uint32_t)((uint64_t)sym_map_cap(cfg) * kFillNum / 100); }
 template <typename V>
 __host__ __device__ inline uint32_t num_map_cap(int cfg) { return (uint32_t)((cfg_map_bytes(cfg) - 16) / num_slot_bytes<V>()); }
 // byte offset of the value array of a numeric hash map (keys first, 16-B aligned values)
@@ -88,11 +113,13 @@ struct BinParams {
   int pass;                 // 0 symbolic, 1 numeric
   int use_direct;           // route single-NZ rows to the direct path
   int64_t cap[kNumCfg];     // need thresholds: row goes to the smallest cfg with need <= cap[cfg]
+  int64_t long_thr;         // numeric: rows with cnt > long_thr are split into segments
 };
 
 __host__ __device__ inline int classify_row(int64_t nnza, int64_t prods, int64_t cnt, const BinParams& bp) {
   if (prods == 0) return CAT_EMPTY;
   if (bp.use_direct && nnza == 1) return CAT_DIRECT;
+  if (bp.pass == 1 && cnt > bp.long_thr) return CAT_LONG;
   int64_t need = bp.pass == 0 ? prods : cnt;
 #pragma unroll
   for (int c = 0; c < kNumCfg - 1; ++c)
@@ -247,6 +274,11 @@ struct SpgemmArgs {
   int64_t resume_stride;
   // counters
   unsigned long long* n_dense_rows;
+  // symbolic, largest configuration: per-chunk counts of long-row candidates
+  int32_t* chunk_cnt;        // [bin entries][nchunks] or nullptr
+  int nchunks;
+  int chunk_shift;           // chunk = col >> chunk_shift
+  int64_t long_thr;          // rows with prods > long_thr record chunk counts
 };
 
 }  // namespace speck

@@ -26,6 +26,7 @@
 namespace speck {
 
 constexpr int kSmallSeg = 64;   // rows with <= this many C entries are ranked, not sorted
+constexpr int kPPL = 4;         // products per lane per chunk in the warp-per-row path
 
 struct BlockMeta {
   int32_t row[kMaxGroupRows];
@@ -35,13 +36,26 @@ struct BlockMeta {
   int32_t cseg[kMaxGroupRows + 1];   // numeric: prefix of cnt_r over the block
   uint32_t rbase[kMaxGroupRows + 1]; // hash region start of each row
   int32_t rcnt[kMaxGroupRows];       // symbolic: distinct columns per row
+  int32_t rg[kMaxGroupRows];         // warp-per-row path: group size per row
+  int32_t rlo[kMaxGroupRows];        // colmin / colmax per row (order-preserving hash)
+  int32_t rhi[kMaxGroupRows];
+  int32_t rwrap[kMaxGroupRows];      // block path: a probing run of the row wrapped around
   uint32_t starts;
-  int nr, g, dense;
+  int nr, g, dense, ordered;
   int64_t nnzA, prods, maxlen, cnt;
   int32_t colmin, colmax;
   int64_t scan_part[33];
   int64_t total;
 };
+
+// every configuration must keep 1024 threads resident per SM: (map + meta + 1 KB) x CTAs/SM
+template <int C>
+constexpr bool cfg_fits() {
+  return (kCfgMapBytes[C] + (int)sizeof(BlockMeta) + 1024) * (1024 / kCfgThreads[C]) <= kSmemPerSM &&
+         kCfgMapBytes[C] + (int)sizeof(BlockMeta) <= kSmemPerCtaMax;
+}
+static_assert(cfg_fits<0>() && cfg_fits<1>() && cfg_fits<2>() && cfg_fits<3>() && cfg_fits<4>(),
+              "a ladder configuration no longer fits 1024 resident threads per SM");
 
 template <typename V>
 __device__ __forceinline__ V ldv(const V* p) { return __ldg(p); }
@@ -59,6 +73,42 @@ __device__ __forceinline__ uint32_t probe_insert(uint32_t* keys, uint32_t S, uin
     }
     s = (s + 1 == S) ? 0u : s + 1;
   }
+}
+
+// Order-preserving home slot for the numeric maps: homes are monotone in the column over the
+// row's [colmin, colmax] and occupy the first 7/8 of the region, the rest absorbs probing
+// runs.  With linear probing and no wrap-around, every key sits in the run ("cluster") that
+// contains its home, and clusters appear in column order; an entry's position in the sorted
+// row is therefore (#occupied slots before its cluster) + (rank of its key inside the cluster).
+__device__ __forceinline__ uint32_t mono_slot(uint32_t col, uint32_t lo, uint32_t range, uint32_t S) {
+  const uint32_t sh = S - (S >> 3);
+  return (uint32_t)(((uint64_t)(col - lo) * sh) / range);
+}
+
+// linear probing that reports a wrap-around (which breaks the cluster order)
+__device__ __forceinline__ uint32_t probe_insert_mono(uint32_t* keys, uint32_t S, uint32_t s, uint32_t key, int* wrapped) {
+  while (true) {
+    const uint32_t k = keys[s];
+    if (k == key) return s;
+    if (k == kEmptyKey) {
+      const uint32_t old = atomicCAS(&keys[s], kEmptyKey, key);
+      if (old == kEmptyKey || old == key) return s;
+    }
+    if (s + 1 == S) { s = 0; *wrapped = 1; } else ++s;
+  }
+}
+
+// Position of the occupied slot s inside its row: `before` = occupied slots before s.
+__device__ __forceinline__ int cluster_position(const uint32_t* keys, uint32_t S, uint32_t s, uint32_t key, int before) {
+  uint32_t cs = s;
+  while (cs > 0 && keys[cs - 1] != kEmptyKey) --cs;
+  int rank = 0;
+  for (uint32_t t = cs; t < S; ++t) {
+    const uint32_t k = keys[t];
+    if (k == kEmptyKey) break;
+    rank += k < key;
+  }
+  return before - (int)(s - cs) + rank;
 }
 
 // symbolic insert: true if the key was new
@@ -79,15 +129,17 @@ __device__ __forceinline__ void hash_accumulate(uint32_t* keys, V* vals, uint32_
 // Bitonic sort of (keys, vals)[0, n) ascending in shared memory, any n: the "flip"
 // formulation keeps all sub-sorts ascending, so comparisons with a partner index >= n
 // (a virtual +inf) are no-ops and can be skipped.
-template <int T, typename V>
+// WARP = true: one warp sorts (lanes 0..31, __syncwarp between stages).
+template <int T, typename V, bool WARP = false>
 __device__ void smem_bitonic_sort(uint32_t* keys, V* vals, int n) {
   if (n <= 1) return;
+  const int t0 = WARP ? (int)(threadIdx.x & 31) : (int)threadIdx.x;
   int P = 1;
   while (P < n) P <<= 1;
   for (int k = 2; k <= P; k <<= 1) {
-    const int hk = k >> 1;
-    for (int t = threadIdx.x; t < P / 2; t += T) {
-      const int blk = t / hk, off = t - blk * hk;
+    const int lhk = __ffs(k) - 2;   // log2(k/2)
+    for (int t = t0; t < P / 2; t += T) {
+      const int blk = t >> lhk, off = t & ((1 << lhk) - 1);
       const int i = blk * k + off, j = blk * k + k - 1 - off;
       if (j < n) {
         const uint32_t a = keys[i], b = keys[j];
@@ -97,11 +149,12 @@ __device__ void smem_bitonic_sort(uint32_t* keys, V* vals, int n) {
         }
       }
     }
-    __syncthreads();
+    if (WARP) __syncwarp(); else __syncthreads();
     for (int d = k >> 2; d >= 1; d >>= 1) {
-      for (int t = threadIdx.x; t < P / 2; t += T) {
-        const int blk = t / d, off = t - blk * d;
-        const int i = blk * 2 * d + off, j = i + d;
+      const int ld = __ffs(d) - 1;
+      for (int t = t0; t < P / 2; t += T) {
+        const int blk = t >> ld, off = t & (d - 1);
+        const int i = (blk << (ld + 1)) + off, j = i + d;
         if (j < n) {
           const uint32_t a = keys[i], b = keys[j];
           if (a > b) {
@@ -110,7 +163,178 @@ __device__ void smem_bitonic_sort(uint32_t* keys, V* vals, int n) {
           }
         }
       }
-      __syncthreads();
+      if (WARP) __syncwarp(); else __syncthreads();
+    }
+  }
+}
+
+// Block-wide write-out of one ordered map region [0, S): warp-contiguous slot ranges, one
+// block scan of the per-warp occupancy, then every entry goes to its sorted position.
+// Contains two block barriers; `part` = >= 32 int64 of shared scratch.
+template <int T, typename V>
+__device__ void block_write_ordered(const uint32_t* rk, const V* rv, uint32_t S, int64_t ob, int32_t* __restrict__ C_col,
+                                    V* __restrict__ C_val, int64_t* part) {
+  constexpr int NW = T / 32;
+  const int lane = lane_id(), wp = warp_id();
+  const uint32_t SW = ((S + NW - 1) / NW + 31u) & ~31u;
+  const uint32_t w0 = min(S, wp * SW), w1 = min(S, w0 + SW);
+  int cw = 0;
+  for (uint32_t c0 = w0; c0 < w1; c0 += 32) {
+    const uint32_t s = c0 + lane;
+    cw += __popc(__ballot_sync(0xffffffffu, s < w1 && rk[s] != kEmptyKey));
+  }
+  if (lane == 0) part[wp] = cw;
+  __syncthreads();
+  int before = 0;
+  for (int w = 0; w < wp; ++w) before += (int)part[w];
+  for (uint32_t c0 = w0; c0 < w1; c0 += 32) {
+    const uint32_t s = c0 + lane;
+    const uint32_t kk = s < w1 ? rk[s] : kEmptyKey;
+    const uint32_t occ = __ballot_sync(0xffffffffu, kk != kEmptyKey);
+    if (kk != kEmptyKey) {
+      const int o = cluster_position(rk, S, s, kk, before + __popc(occ & ((1u << lane) - 1u)));
+      C_col[ob + o] = (int32_t)kk;
+      C_val[ob + o] = rv[s];
+    }
+    before += __popc(occ);
+  }
+  __syncthreads();
+}
+
+// Sum of v over the lanes of the warp holding the same key (all 32 lanes call it; keys of
+// inactive lanes must be unique).  `leader` = lowest lane of its key group, which receives
+// the sum — so one update per distinct key per warp step instead of one atomic per product.
+template <typename V>
+__device__ __forceinline__ V warp_key_sum(uint32_t key, V v, bool& leader) {
+  const int lane = lane_id();
+  const uint32_t peers = __match_any_sync(0xffffffffu, key);
+  leader = lane == __ffs(peers) - 1;
+  const int maxg = (int)__reduce_max_sync(0xffffffffu, (unsigned)__popc(peers));
+  V sum = v;
+  if (maxg > 1) {
+    uint32_t others = leader ? (peers & ~(1u << lane)) : 0u;
+    for (int t = 1; t < maxg; ++t) {
+      int src = lane;
+      if (others) { src = __ffs(others) - 1; others &= others - 1; }
+      const V x = __shfl_sync(0xffffffffu, v, src);
+      if (src != lane) sum += x;
+    }
+  }
+  return sum;
+}
+
+// Expand-balanced local load balancing (B200 form of the paper's local load balancer,
+// P:867-970, which calls exact per-entry balancing ideal but too costly).
+// Products of a row of A are enumerated in batches of 32 referenced B rows (one per lane:
+// A col -> B row start/length), a warp scan of the lengths, then every lane takes products
+// lane, lane+32, ... located by a 5-step shuffle binary search, kPPL per lane per chunk with
+// independent loads (memory-level parallelism).  `nw` warps (index wi) share a row: a single
+// batch splits its product chunks across the warps, several batches go round-robin.
+// ins(col, val, active) is called by all 32 lanes (inactive lanes get a unique non-column key).
+// Variant with a per-referenced-row sub-range: rng(f, j0, j1, s, e) narrows B row [j0, j1)
+// of the f-th NZ of the row of A to [s, e) (column windows / segments); called once per f.
+struct FullRange {
+  __device__ __forceinline__ void operator()(int, int64_t j0, int64_t j1, int64_t& s, int64_t& e) const { s = j0; e = j1; }
+};
+
+template <int PASS, typename V, typename Ins, typename Rng = FullRange>
+__device__ __forceinline__ void expand_row(const SpgemmArgs<V>& p, int64_t a0, int alen, int wi, int nw, Ins&& ins,
+                                           Rng rng = Rng()) {
+  const int lane = lane_id();
+  const int nb = (alen + 31) >> 5;
+  const bool share = nb == 1;
+  constexpr int CH = 32 * kPPL;
+  for (int b = share ? 0 : wi; b < nb; b += share ? 1 : nw) {
+    const int f = b * 32 + lane;
+    int64_t bst = 0;
+    int blen = 0;
+    V a = V(0);
+    if (f < alen) {
+      const int32_t kc = p.A_col[a0 + f];
+      if (PASS == 1) a = ldv(p.A_val + a0 + f);
+      int64_t s, e;
+      rng(f, p.B_rp[kc], p.B_rp[kc + 1], s, e);
+      bst = s;
+      blen = (int)(e - s);
+    }
+    const int incl = warp_incl_scan(blen);
+    const int excl = incl - blen;
+    const int Pb = __shfl_sync(0xffffffffu, incl, 31);
+    for (int p0 = (share ? wi : 0) * CH; p0 < Pb; p0 += (share ? nw : 1) * CH) {
+      uint32_t col[kPPL];
+      V v[kPPL];
+#pragma unroll
+      for (int i = 0; i < kPPL; ++i) {
+        const int pp = p0 + lane + 32 * i;
+        int lo = 0;   // owner lane: smallest o with incl_o > pp
+#pragma unroll
+        for (int step = 16; step > 0; step >>= 1) {
+          const int probe = __shfl_sync(0xffffffffu, incl, lo + step - 1);
+          if (probe <= pp) lo += step;
+        }
+        const int o = lo > 31 ? 31 : lo;
+        const int64_t idx = __shfl_sync(0xffffffffu, bst, o) + (pp - __shfl_sync(0xffffffffu, excl, o));
+        const V ao = PASS == 1 ? __shfl_sync(0xffffffffu, a, o) : V(0);
+        col[i] = 0x80000000u | (uint32_t)lane;   // inactive: never a real column (< 2^31)
+        v[i] = V(0);
+        if (pp < Pb) {
+          col[i] = (uint32_t)p.B_col[idx];
+          if (PASS == 1) v[i] = ao * ldv(p.B_val + idx);
+        }
+      }
+#pragma unroll
+      for (int i = 0; i < kPPL; ++i) ins(col[i], v[i], p0 + lane + 32 * i < Pb);
+    }
+  }
+}
+
+// first index in [l, h) with col >= x (rows of B are sorted)
+__device__ __forceinline__ int64_t lower_bound_col(const int32_t* __restrict__ col, int64_t l, int64_t h, uint32_t x) {
+  while (l < h) {
+    const int64_t mid = (l + h) >> 1;
+    if ((uint32_t)col[mid] < x) l = mid + 1; else h = mid;
+  }
+  return l;
+}
+
+// Column windows processed in ascending order: each referenced B row resumes where the
+// previous window stopped and ends at the first column >= whi.  The resume
+// offsets are double-buffered (read cur, write next; the caller swaps after the window's
+// barrier), because warps sharing one batch of a row all evaluate the same f.
+struct WindowRange {
+  const int32_t* cur;        // resume offsets per NZ of the row of A (relative to the B row start)
+  int32_t* next;
+  const int32_t* bcol;
+  uint32_t whi;
+  __device__ __forceinline__ void operator()(int f, int64_t j0, int64_t j1, int64_t& s, int64_t& e) const {
+    s = j0 + cur[f];
+    e = lower_bound_col(bcol, s, j1, whi);
+    next[f] = (int32_t)(e - j0);
+  }
+};
+
+// An independent column range [lo, hi) of every referenced B row (long-row segments).
+struct SegRange {
+  const int32_t* bcol;
+  uint32_t lo, hi;
+  __device__ __forceinline__ void operator()(int, int64_t j0, int64_t j1, int64_t& s, int64_t& e) const {
+    s = lower_bound_col(bcol, j0, j1, lo);
+    e = lower_bound_col(bcol, s, j1, hi);
+  }
+};
+
+// Dense-window insert: flag bit (structural entry) and, numeric, the value (warp-aggregated).
+template <int PASS, typename V>
+__device__ __forceinline__ void dense_insert(uint32_t* bits, V* dvals, uint32_t wlo, uint32_t col, V v, bool act) {
+  const uint32_t c = col - wlo;
+  if (PASS == 0) {
+    if (act) atomicOr(&bits[c >> 5], 1u << (c & 31));
+  } else {
+    bool leader;
+    const V sum = warp_key_sum(col, v, leader);
+    if (act && leader) {
+      atomicOr(&bits[c >> 5], 1u << (c & 31));
+      atomicAdd(&dvals[c], sum);
     }
   }
 }
@@ -131,6 +355,7 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
   
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ BlockMeta bm;
+  __shared__ int chist[(CFG == kNumCfg - 1 && PASS == 0) ? kMaxChunks : 1];
   const int tid = threadIdx.x;
 
   const int64_t e0 = (int64_t)blockIdx.x * p.group_rows;
@@ -189,6 +414,7 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
       uint32_t rsz = 0;
       if (l < nr) rsz = nr == 1 ? cap : (need_tot > 0 ? (uint32_t)((uint64_t)cap * (uint64_t)need / (uint64_t)need_tot) : 0u);
       const uint32_t rinc = warp_incl_scan(rsz);
+      const bool any_small = __any_sync(0xffffffffu, l < nr && c <= kSmallSeg);
       if (l < nr) {
         bm.astart[l] = a0;
         bm.aoff[l + 1] = ainc;
@@ -196,10 +422,16 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
         bm.cseg[l + 1] = (int32_t)cinc;
         bm.rbase[l + 1] = rinc;
         bm.rcnt[l] = 0;
+        bm.rlo[l] = cmn;
+        bm.rhi[l] = cmx;
+        bm.rwrap[l] = 0;
+        // per-row group size for the warp-per-row path (local LB with T = one warp)
+        bm.rg[l] = p.fixed_g > 0 ? min(p.fixed_g, 32) : local_group_size(32, alen, pr, ml);
       }
       if (l == 0) {
         bm.aoff[0] = 0; bm.cseg[0] = 0; bm.rbase[0] = 0;
         bm.nr = nr;
+        bm.ordered = PASS == 1 && !any_small;
         bm.nnzA = tot_a;
         bm.prods = tot_p;
         bm.maxlen = mlx;
@@ -213,7 +445,7 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
           if (PASS == 0) {
             const int64_t W = sym_dense_window(CFG);
             if (p.force_acc == 2) dense = 1;
-            else if ((uint64_t)tot_p > (uint64_t)cap) dense = 1;                       // cannot hash: P:1112-1113
+            else if ((uint64_t)tot_p > (uint64_t)sym_map_fill(CFG)) dense = 1;         // beyond the map: P:1112-1113
             else if (p.force_acc != 1 && range <= W && range <= 16 * tot_p) dense = 1;  // bitmap cheaper than hashing
           } else {
             const int64_t W = num_dense_window<V>(CFG);
@@ -231,22 +463,113 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
           }
         }
         bm.dense = dense;
-        // ---- local load balancer ----
-        int g = p.fixed_g > 0 ? min(p.fixed_g, T) : local_group_size(T, tot_a, tot_p, mlx);
-        if (dense) {
-          const int64_t W0 = PASS == 0 ? sym_dense_window(CFG) : num_dense_window<V>(CFG);
-          const int64_t W = (p.dense_window_cap > 0 && p.dense_window_cap < W0) ? p.dense_window_cap : W0;
-          if (range > W && g > 32) g = 32;  // multi-window rows: a group must fit a warp
-        }
-        bm.g = g;
       }
     }
     __syncthreads();
-    const int g = bm.g;
-    const int gid = tid / g, gl = tid - gid * g, k = T / g;
     const int64_t nnzA = bm.nnzA;
+    constexpr int NW = T / 32;
 
-    if (!bm.dense) {
+    if (!bm.dense && nr >= NW && nr > 1) {
+      // ===================== HASH, WARP PER ROW (multi-row blocks) =====================
+      // Each warp owns whole rows and their private map regions, so accumulation and the
+      // sort/compaction epilogue need no block barrier; lanes whose key is unique within
+      // the warp step update the value with a plain read-modify-write.
+      uint32_t* keys = reinterpret_cast<uint32_t*>(smem);
+      V* vals = reinterpret_cast<V*>(smem + (PASS == 0 ? 0u : num_val_offset<V>(CFG)));
+      const int lane = lane_id();
+      for (int r = warp_id(); r < nr; r += NW) {
+        const uint32_t rb = bm.rbase[r], S = bm.rbase[r + 1] - rb;
+        uint32_t* rk = keys + rb;
+        V* rv = vals + rb;
+        for (uint32_t i = lane; i < S; i += 32) {
+          rk[i] = kEmptyKey;
+          if (PASS == 1) rv[i] = V(0);
+        }
+        __syncwarp();
+        const int64_t a0 = bm.astart[r];
+        const int alen = (int)(bm.aoff[r + 1] - bm.aoff[r]);
+        const uint32_t mlo = (uint32_t)bm.rlo[r];
+        const uint32_t mrange = (uint32_t)(bm.rhi[r] - bm.rlo[r] + 1);
+        // long rows use the order-preserving map (sorted write-out without a sort network);
+        // short rows keep the scrambled hash (robust to clustered columns) and rank counting
+        const bool ordered = PASS == 1 && bm.cseg[r + 1] - bm.cseg[r] > kSmallSeg;
+        int newc = 0, wrapped = 0;
+        expand_row<PASS, V>(p, a0, alen, 0, 1, [&](uint32_t col, V v, bool act) {
+          if (PASS == 0) {
+            if (act) newc += hash_insert_key(rk, S, col);
+          } else {
+            uint32_t s = 0;
+            if (act)
+              s = probe_insert_mono(rk, S, ordered ? mono_slot(col, mlo, mrange, S) : hash_slot(col, S), col, &wrapped);
+            bool leader;
+            const V sum = warp_key_sum(col, v, leader);
+            if (act && leader) rv[s] += sum;   // the region is private to this warp: no atomic
+            __syncwarp();
+          }
+        });
+        if (PASS == 0) {
+          newc = warp_sum(newc);
+          if (lane == 0) p.cnt[bm.row[b0 + r]] = newc;
+        } else if (ordered && !__any_sync(0xffffffffu, wrapped)) {
+          // ordered map: write every entry at (occupied slots before its cluster) + (rank in
+          // the cluster) — the row comes out sorted without moving anything in shared memory
+          const int64_t ob = bm.cbase[r];
+          int before = 0;
+          for (uint32_t c0 = 0; c0 < S; c0 += 32) {
+            const uint32_t s = c0 + lane;
+            const uint32_t kk = s < S ? rk[s] : kEmptyKey;
+            const uint32_t occ = __ballot_sync(0xffffffffu, kk != kEmptyKey);
+            if (kk != kEmptyKey) {
+              const int o = cluster_position(rk, S, s, kk, before + __popc(occ & ((1u << lane) - 1u)));
+              p.C_col[ob + o] = (int32_t)kk;
+              p.C_val[ob + o] = rv[s];
+            }
+            before += __popc(occ);
+          }
+        } else {
+          // a probing run wrapped around: compact the region in place, then sort and write
+          int pos = 0;
+          for (uint32_t c0 = 0; c0 < S; c0 += 32) {
+            const uint32_t s = c0 + lane;
+            uint32_t kk = kEmptyKey;
+            V vv = V(0);
+            if (s < S) { kk = rk[s]; vv = rv[s]; }
+            const uint32_t occ = __ballot_sync(0xffffffffu, kk != kEmptyKey);
+            __syncwarp();
+            if (kk != kEmptyKey) {
+              const int o = pos + __popc(occ & ((1u << lane) - 1u));
+              rk[o] = kk;
+              rv[o] = vv;
+            }
+            pos += __popc(occ);
+            __syncwarp();
+          }
+          const int cnt = pos;
+          const int64_t ob = bm.cbase[r];
+          if (cnt <= kSmallSeg) {
+            // rank counting: all lanes read key j together (smem broadcast)
+            for (int e0 = 0; e0 < cnt; e0 += 32) {
+              const int e = e0 + lane;
+              const uint32_t key = e < cnt ? rk[e] : 0xffffffffu;
+              const V val = e < cnt ? rv[e] : V(0);
+              int rank = 0;
+              for (int j = 0; j < cnt; ++j) rank += rk[j] < key;
+              if (e < cnt) {
+                p.C_col[ob + rank] = (int32_t)key;
+                p.C_val[ob + rank] = val;
+              }
+            }
+          } else {
+            smem_bitonic_sort<32, V, true>(rk, rv, cnt);
+            for (int e = lane; e < cnt; e += 32) {
+              p.C_col[ob + e] = (int32_t)rk[e];
+              p.C_val[ob + e] = rv[e];
+            }
+          }
+        }
+        __syncwarp();
+      }
+    } else if (!bm.dense) {
       // ============================ HASH ACCUMULATOR ==============================
       uint32_t* keys = reinterpret_cast<uint32_t*>(smem);
       const uint32_t capt = bm.rbase[nr];
@@ -256,26 +579,61 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
         if (PASS == 1) vals[i] = V(0);
       }
       __syncthreads();
-      int r = 0;
-      for (int64_t f = gid; f < nnzA; f += k) {
-        while (f >= bm.aoff[r + 1]) ++r;
-        const int64_t q = bm.astart[r] + (f - bm.aoff[r]);
-        const int32_t kc = p.A_col[q];
-        const int64_t j0 = p.B_rp[kc], j1 = p.B_rp[kc + 1];
+      // all warps share each row: expand-balanced products, warp aggregation of equal keys,
+      // one atomic per distinct key per warp step (other warps may hold the same key)
+      for (int r = 0; r < nr; ++r) {
         const uint32_t rb = bm.rbase[r], S = bm.rbase[r + 1] - rb;
+        uint32_t* rk = keys + rb;
+        V* rv = vals + rb;
+        const uint32_t mlo = (uint32_t)bm.rlo[r], mrange = (uint32_t)(bm.rhi[r] - bm.rlo[r] + 1);
+        const bool ordered = bm.ordered;
+        int newc = 0, wrapped = 0;
+        expand_row<PASS, V>(p, bm.astart[r], (int)(bm.aoff[r + 1] - bm.aoff[r]), warp_id(), NW,
+                            [&](uint32_t col, V v, bool act) {
+                              if (PASS == 0) {
+                                if (act) newc += hash_insert_key(rk, S, col);
+                              } else {
+                                uint32_t s = 0;
+                                if (act)
+                                  s = probe_insert_mono(rk, S, ordered ? mono_slot(col, mlo, mrange, S) : hash_slot(col, S),
+                                                        col, &wrapped);
+                                bool leader;
+                                const V sum = warp_key_sum(col, v, leader);
+                                if (act && leader) atomicAdd(&rv[s], sum);
+                              }
+                            });
         if (PASS == 0) {
-          int newc = 0;
-          for (int64_t j = j0 + gl; j < j1; j += g) newc += hash_insert_key(keys + rb, S, (uint32_t)p.B_col[j]);
-          if (newc) atomicAdd(&bm.rcnt[r], newc);
-        } else {
-          const V a = ldv(p.A_val + q);
-          for (int64_t j = j0 + gl; j < j1; j += g)
-            hash_accumulate<V>(keys + rb, vals + rb, S, (uint32_t)p.B_col[j], a * ldv(p.B_val + j));
+          newc = warp_sum(newc);
+          if (lane_id() == 0 && newc) atomicAdd(&bm.rcnt[r], newc);
+        } else if (__any_sync(0xffffffffu, wrapped) && lane_id() == 0) {
+          bm.rwrap[r] = 1;
         }
       }
       __syncthreads();
+      int any_wrap = !bm.ordered;   // scrambled maps take the compaction + sort epilogue
+      if (PASS == 1)
+        for (int rr = 0; rr < nr; ++rr) any_wrap |= bm.rwrap[rr];
       if (PASS == 0) {
         if (tid < nr) p.cnt[bm.row[b0 + tid]] = bm.rcnt[tid];
+        if (CFG == kNumCfg - 1 && p.chunk_cnt && nr == 1 && bm.prods > p.long_thr) {
+          // long-row candidate: distinct columns per 2^15-column chunk, for the numeric split
+          for (int i = tid; i < p.nchunks; i += T) chist[i] = 0;
+          __syncthreads();
+          for (uint32_t s = tid; s < capt; s += T) {
+            const uint32_t kk = keys[s];
+            if (kk != kEmptyKey) atomicAdd(&chist[kk >> p.chunk_shift], 1);
+          }
+          __syncthreads();
+          int32_t* dst = p.chunk_cnt + (int64_t)blockIdx.x * p.nchunks;
+          for (int i = tid; i < p.nchunks; i += T) dst[i] = chist[i];
+        }
+      } else if (!any_wrap) {
+        // ---- ordered maps: each entry goes to (occupied before its cluster) + (rank in it) ----
+        for (int rr = 0; rr < nr; ++rr) {
+          const uint32_t rb = bm.rbase[rr];
+          block_write_ordered<T, V>(keys + rb, vals + rb, bm.rbase[rr + 1] - rb, bm.cbase[rr], p.C_col, p.C_val,
+                                    bm.scan_part);
+        }
       } else {
         // ---- compaction (order preserving -> row regions stay in row order) ----
         int64_t running = 0;
@@ -324,20 +682,26 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
       // ============================ DENSE ACCUMULATOR =============================
       // single row; windows over [colmin, colmax] (Fig. 5)
       const int32_t row = bm.row[b0];
-      const int64_t lo = bm.colmin, hi = bm.colmax;
+      // symbolic windows start 32-aligned so a bitmap word never straddles a 2^15 chunk
+      const int64_t lo = PASS == 0 ? (bm.colmin & ~31) : bm.colmin, hi = bm.colmax;
+      const bool chunks = CFG == kNumCfg - 1 && PASS == 0 && p.chunk_cnt && bm.prods > p.long_thr;
+      if (chunks) {
+        for (int i = tid; i < p.nchunks; i += T) chist[i] = 0;   // ordered by the window's barrier
+      }
       const int64_t W0 = PASS == 0 ? sym_dense_window(CFG) : num_dense_window<V>(CFG);
       const int64_t W = (p.dense_window_cap > 0 && p.dense_window_cap < W0) ? p.dense_window_cap : W0;
       const int64_t nwin = (hi - lo + 1 + W - 1) / W;
       const int64_t astart = bm.astart[0];
       uint32_t* bits = reinterpret_cast<uint32_t*>(smem);                       // W bits
       V* dvals = reinterpret_cast<V*>(smem + (PASS == 0 ? 0 : (((W + 31) / 32) * 4 + 15) / 16 * 16));
-      int32_t* res = nullptr;
+      int32_t* res = nullptr;       // double-buffered resume offsets (cur, next)
+      int32_t* res_next = nullptr;
       if (nwin > 1) {
         res = p.resume + (int64_t)smid() * p.resume_stride;
+        res_next = res + p.resume_stride / 2;
         for (int64_t f = tid; f < nnzA; f += T) res[f] = 0;
       }
       const int nwords = (int)((W + 31) / 32);
-      const uint32_t gmask = g >= 32 ? 0xffffffffu : (((1u << g) - 1u) << (lane_id() & ~(g - 1)));
       int64_t out = PASS == 1 ? bm.cbase[0] : 0;
       int64_t total = 0;
       if (tid == 0 && PASS == 1 && p.n_dense_rows) atomicAdd(p.n_dense_rows, 1ull);
@@ -347,38 +711,12 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
         if (PASS == 1)
           for (int64_t i = tid; i < W; i += T) dvals[i] = V(0);
         __syncthreads();
-        for (int64_t f = gid; f < nnzA; f += k) {
-          const int64_t q = astart + f;
-          const int32_t kc = p.A_col[q];
-          const int64_t j0 = p.B_rp[kc], j1 = p.B_rp[kc + 1];
-          V a = V(0);
-          if (PASS == 1) a = ldv(p.A_val + q);
-          if (nwin == 1) {
-            for (int64_t j = j0 + gl; j < j1; j += g) {
-              const uint32_t c = (uint32_t)(p.B_col[j] - wlo);
-              atomicOr(&bits[c >> 5], 1u << (c & 31));
-              if (PASS == 1) atomicAdd(&dvals[c], a * ldv(p.B_val + j));
-            }
-          } else {
-            int64_t pos = j0 + res[f];
-            while (pos < j1) {
-              const int64_t j = pos + gl;
-              const int32_t cj = j < j1 ? p.B_col[j] : 0x7fffffff;
-              const bool in = cj < whi;
-              if (in) {
-                const uint32_t c = (uint32_t)(cj - wlo);
-                atomicOr(&bits[c >> 5], 1u << (c & 31));
-                if (PASS == 1) atomicAdd(&dvals[c], a * ldv(p.B_val + j));
-              }
-              const uint32_t bal = __ballot_sync(gmask, in);
-              const int took = __popc(bal);
-              pos += took;
-              if (took < g) break;
-            }
-            if (gl == 0) res[f] = (int32_t)(pos - j0);
-          }
-        }
+        // expand-balanced accumulation of the products falling into this window
+        auto ins = [&](uint32_t col, V v, bool act) { dense_insert<PASS, V>(bits, dvals, (uint32_t)wlo, col, v, act); };
+        if (nwin == 1) expand_row<PASS, V>(p, astart, (int)nnzA, warp_id(), NW, ins);
+        else expand_row<PASS, V>(p, astart, (int)nnzA, warp_id(), NW, ins, WindowRange{res, res_next, p.B_col, (uint32_t)whi});
         __syncthreads();
+        { int32_t* t_ = res; res = res_next; res_next = t_; }
         // ---- window epilogue: count (symbolic) / compact in column order (numeric) ----
         int64_t wtot = 0;
         for (int base = 0; base < nwords; base += T) {
@@ -387,6 +725,7 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
           const int64_t pc = __popc(word);
           int64_t tot;
           const int64_t pre = block_excl_scan<T>(pc, bm.scan_part, &tot);
+          if (PASS == 0 && chunks && word) atomicAdd(&chist[(wlo + (int64_t)wi * 32) >> p.chunk_shift], (int)pc);
           if (PASS == 1 && word) {
             uint32_t wd = word;
             int64_t o = out + wtot + pre;
@@ -406,6 +745,10 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
         __syncthreads();
       }
       if (PASS == 0 && tid == 0) p.cnt[row] = total;
+      if (chunks) {
+        int32_t* dst = p.chunk_cnt + (int64_t)blockIdx.x * p.nchunks;
+        for (int i = tid; i < p.nchunks; i += T) dst[i] = chist[i];
+      }
     }
     __syncthreads();
     b0 = b1;

@@ -23,6 +23,7 @@ SPECK_F32, SPECK_F64 = 0, 1
 OPT = {
     "global_lb_symbolic": 0, "global_lb_numeric": 1, "force_accumulator": 2, "dense_window": 3,
     "stage_timing": 4, "validate": 5, "disable_direct": 6, "fixed_group_size": 7, "concurrent_streams": 8,
+    "segments": 9,
 }
 STATUS = {
     0: "SPECK_OK", 1: "SPECK_ERR_INVALID_ARGUMENT", 2: "SPECK_ERR_DIMENSION_MISMATCH", 3: "SPECK_ERR_DTYPE_MISMATCH",
@@ -54,6 +55,7 @@ class Stats(ctypes.Structure):
                 ("rows_direct", ctypes.c_int64), ("rows_empty", ctypes.c_int64), ("lb_symbolic", ctypes.c_int32),
                 ("lb_numeric", ctypes.c_int32), ("rows_per_bin_symbolic", ctypes.c_int64 * 8),
                 ("rows_per_bin_numeric", ctypes.c_int64 * 8), ("rows_dense_numeric", ctypes.c_int64),
+                ("segments", ctypes.c_int64),
                 ("workspace_bytes", ctypes.c_int64), ("kernel_launches", ctypes.c_int64), ("ms_analysis", ctypes.c_float), ("ms_symbolic_lb", ctypes.c_float),
                 ("ms_symbolic", ctypes.c_float), ("ms_scan", ctypes.c_float), ("ms_numeric_lb", ctypes.c_float),
                 ("ms_numeric", ctypes.c_float)]

@@ -189,6 +189,28 @@ def test_path_forcing_same_result(dev, opts):
     assert_parity(A2, B2, C2)
 
 
+@pytest.mark.parametrize("segments", [1, 0])
+@pytest.mark.parametrize("dt", [torch.float32, torch.float64])
+def test_long_rows(dev, segments, dt):
+    """Rows of C beyond the largest hash map: dense-ish (~100% of a 200k range) and sparse
+    (~5% of a 2M range) long rows — column segments (default) or windowed dense."""
+    A = W.random_sparse(6, 2000, 0.5, seed=31, dtype=dt)
+    B = W.random_sparse(2000, 200_000, 0.01, seed=32, dtype=dt)
+    C, st = gpu_spgemm(A, B, segments=segments)
+    assert_parity(A, B, C)
+    if segments:
+        assert st["segments"] > 0 and st["rows_per_bin_numeric"][7] == 6
+    import numpy as _np
+    rng = _np.random.default_rng(3)
+    # sparse long rows: 2000 B rows x 50 random columns of 2M
+    cols = torch.tensor(_np.sort(rng.choice(2_000_000, size=(2000, 50), replace=True), axis=1).astype(_np.int64))
+    r = torch.arange(2000).repeat_interleave(50)
+    B2 = W.csr_from_coo(2000, 2_000_000, r, cols.reshape(-1), None, dtype=dt, seed=5)
+    A2 = W.random_sparse(4, 2000, 0.9, seed=33, dtype=dt)
+    C2, st2 = gpu_spgemm(A2, B2, segments=segments)
+    assert_parity(A2, B2, C2)
+
+
 def test_fig5_dense_window_of_three(dev):
     """Fig. 5: one row, 6 columns, window 3, products at c0,c2,c4,c4,c5 -> c0=1 c2=1 c4=2 c5=1."""
     kv, _ = golden("fig5_dense.txt")
