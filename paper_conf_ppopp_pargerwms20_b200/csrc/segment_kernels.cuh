@@ -59,16 +59,27 @@ struct SegPlanArgs {
   int shift;
   int64_t limit;           // numeric long-row threshold = entries of a hashed segment
   int64_t dense_window;    // columns of one dense window of the largest configuration
+  int64_t map_slots;       // slots of the largest numeric hash map
   int prefer_parallel;     // few long rows: always split (parallelism across SMs)
 };
 
-// A row is processed as one "windows" job when its windows cost little next to its products:
-// #windows · nnz(A_i) <= products (each window revisits every referenced B row once).
-__device__ __forceinline__ bool use_windows(const SegPlanArgs& a, int32_t row) {
+// One "windows" job or column segments for a long row: estimated per-row overheads (the
+// products themselves cost the same either way).  Windows: per window, clear + scan the dense
+// array and revisit every referenced B row (resume position + one binary search).  Segments:
+// per segment, two binary searches per referenced B row and a map clear.  With few long rows
+// the row is always split so its work spreads over the SMs.
+__device__ __forceinline__ bool use_windows(const SegPlanArgs& a, int32_t row, int64_t cnt, int64_t map_slots) {
   if (a.prefer_parallel) return false;
   const int64_t range = (int64_t)a.colmax[row] - a.colmin[row] + 1;
   const int64_t nwin = (range + a.dense_window - 1) / a.dense_window;
-  return nwin * (a.A_rp[row + 1] - a.A_rp[row]) <= a.prods[row];
+  const int64_t dA = a.A_rp[row + 1] - a.A_rp[row];
+  const int64_t avg = dA > 0 ? a.prods[row] / dA + 1 : 1;
+  int64_t lg = 1;
+  while ((int64_t)1 << lg < avg) ++lg;
+  const int64_t nseg = cnt / a.limit + 1;
+  const int64_t win_cost = nwin * (a.dense_window / 8 + dA * (1 + lg));
+  const int64_t seg_cost = nseg * (dA * 2 * lg + map_slots / 4);
+  return win_cost <= seg_cost;
 }
 
 // Pass 1: number of jobs of every long-row candidate (one thread per candidate).
@@ -79,7 +90,7 @@ __global__ void k_seg_count(SegPlanArgs a, int64_t* __restrict__ nseg) {
   const int64_t cnt = a.C_rp[row + 1] - a.C_rp[row];
   int64_t n = 0;
   if (cnt > a.limit) {
-    if (use_windows(a, row)) {
+    if (use_windows(a, row, cnt, a.map_slots)) {
       n = 1;
     } else {
       plan_row_segments(a.chunk_cnt + e * a.nchunks, a.colmin[row] >> a.shift, a.colmax[row] >> a.shift, a.limit,
@@ -99,7 +110,7 @@ __global__ void k_seg_emit(SegPlanArgs a, const int64_t* __restrict__ seg_off, S
   if (cnt <= a.limit) return;
   const int32_t lo = a.colmin[row], hi = a.colmax[row];
   int64_t o = seg_off[e];
-  if (use_windows(a, row)) {
+  if (use_windows(a, row, cnt, a.map_slots)) {
     Seg s;
     s.row = row; s.col_lo = lo; s.col_hi = hi + 1; s.cnt = (int32_t)(cnt < 0x7fffffff ? cnt : 0x7fffffff); s.out = c0;
     s.dense = SEG_WINDOWS; s.pad = 0;
@@ -140,26 +151,7 @@ __device__ int64_t dense_window_pass(const SpgemmArgs<V>& p, int64_t a0, int ale
   expand_row<1, V>(p, a0, alen, warp_id(), NW,
                    [&](uint32_t col, V v, bool act) { dense_insert<1, V>(bits, dvals, wlo, col, v, act); }, rng);
   __syncthreads();
-  int64_t done = 0;
-  for (int base = 0; base < nwords; base += T) {
-    const int wi = base + tid;
-    const uint32_t word = wi < nwords ? bits[wi] : 0u;
-    int64_t tot;
-    const int64_t pre = block_excl_scan<T>((int64_t)__popc(word), part, &tot);
-    uint32_t wd = word;
-    int64_t o = out + done + pre;
-    while (wd) {
-      const int b = __ffs(wd) - 1;
-      wd &= wd - 1;
-      const uint32_t ci = (uint32_t)wi * 32 + b;
-      p.C_col[o] = (int32_t)(wlo + ci);
-      p.C_val[o] = dvals[ci];
-      ++o;
-    }
-    done += tot;
-  }
-  __syncthreads();
-  return done;
+  return dense_emit<T, V>(bits, dvals, nwords, wlo, out, p.C_col, p.C_val, part);
 }
 
 // One CTA (the largest configuration, 1 CTA/SM) per job.

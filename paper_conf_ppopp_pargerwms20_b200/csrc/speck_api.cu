@@ -320,6 +320,7 @@ SegPlanArgs seg_plan_args(speck_handle_t h, const int64_t* C_rp) {
   s.shift = h->seg_shift;
   s.limit = h->long_thr;
   s.dense_window = num_dense_window<V>(kNumCfg - 1);
+  s.map_slots = num_map_cap<V>(kNumCfg - 1);
   // few candidates: split every long row so its work spreads over the SMs
   s.prefer_parallel = h->n_cand < 4 * (int64_t)h->num_sms ? 1 : 0;
   return s;

@@ -242,9 +242,14 @@ __device__ __forceinline__ void expand_row(const SpgemmArgs<V>& p, int64_t a0, i
                                            Rng rng = Rng()) {
   const int lane = lane_id();
   const int nb = (alen + 31) >> 5;
-  const bool share = nb == 1;
   constexpr int CH = 32 * kPPL;
-  for (int b = share ? 0 : wi; b < nb; b += share ? 1 : nw) {
+  // fewer batches than warps: G = nw/nb warps per batch, splitting its product chunks;
+  // otherwise batches go round-robin and a warp takes all chunks of its batch
+  const int G = nb >= nw ? 1 : nw / nb;
+  const bool share = G > 1;
+  const int b_first = share ? wi / G : wi, b_step = share ? nb : nw;   // share: one batch per warp group
+  const int c_first = share ? wi % G : 0, c_step = share ? G : 1;
+  for (int b = b_first; b < nb; b += b_step) {
     const int f = b * 32 + lane;
     int64_t bst = 0;
     int blen = 0;
@@ -260,11 +265,14 @@ __device__ __forceinline__ void expand_row(const SpgemmArgs<V>& p, int64_t a0, i
     const int incl = warp_incl_scan(blen);
     const int excl = incl - blen;
     const int Pb = __shfl_sync(0xffffffffu, incl, 31);
-    for (int p0 = (share ? wi : 0) * CH; p0 < Pb; p0 += (share ? nw : 1) * CH) {
+    for (int p0 = c_first * CH; p0 < Pb; p0 += c_step * CH) {
       uint32_t col[kPPL];
       V v[kPPL];
 #pragma unroll
       for (int i = 0; i < kPPL; ++i) {
+        col[i] = 0x80000000u | (uint32_t)lane;
+        v[i] = V(0);
+        if (p0 + 32 * i >= Pb) continue;   // warp-uniform: the whole sub-chunk is past the row
         const int pp = p0 + lane + 32 * i;
         int lo = 0;   // owner lane: smallest o with incl_o > pp
 #pragma unroll
@@ -275,15 +283,14 @@ __device__ __forceinline__ void expand_row(const SpgemmArgs<V>& p, int64_t a0, i
         const int o = lo > 31 ? 31 : lo;
         const int64_t idx = __shfl_sync(0xffffffffu, bst, o) + (pp - __shfl_sync(0xffffffffu, excl, o));
         const V ao = PASS == 1 ? __shfl_sync(0xffffffffu, a, o) : V(0);
-        col[i] = 0x80000000u | (uint32_t)lane;   // inactive: never a real column (< 2^31)
-        v[i] = V(0);
-        if (pp < Pb) {
+        if (pp < Pb) {   // inactive lanes keep a key that is never a real column (< 2^31)
           col[i] = (uint32_t)p.B_col[idx];
           if (PASS == 1) v[i] = ao * ldv(p.B_val + idx);
         }
       }
 #pragma unroll
-      for (int i = 0; i < kPPL; ++i) ins(col[i], v[i], p0 + lane + 32 * i < Pb);
+      for (int i = 0; i < kPPL; ++i)
+        if (p0 + 32 * i < Pb) ins(col[i], v[i], p0 + lane + 32 * i < Pb);   // uniform skip of empty sub-chunks
     }
   }
 }
@@ -337,6 +344,51 @@ __device__ __forceinline__ void dense_insert(uint32_t* bits, V* dvals, uint32_t 
       atomicAdd(&dvals[c], sum);
     }
   }
+}
+
+// Coalesced, sorted write-out of a numeric dense window (values + flag bits): warp w owns a
+// contiguous range of flag words; pass 1 counts, one block-level prefix over the warps, pass 2
+// broadcasts each word and lane b writes the entry of bit b, so every store instruction
+// writes up to 32 consecutive entries of C.  Returns the entries written (barriers inside).
+template <int T, typename V>
+__device__ int64_t dense_emit(const uint32_t* bits, const V* dvals, int nwords, uint32_t wlo, int64_t out,
+                              int32_t* __restrict__ C_col, V* __restrict__ C_val, int64_t* part) {
+  constexpr int NW = T / 32;
+  const int lane = lane_id(), wp = warp_id();
+  const int WW = ((nwords + NW - 1) / NW + 31) & ~31;
+  const int w0 = min(nwords, wp * WW), w1 = min(nwords, w0 + WW);
+  int cnt = 0;
+  for (int i = w0 + lane; i < w1; i += 32) cnt += __popc(bits[i]);
+  cnt = warp_sum(cnt);
+  if (lane == 0) part[wp] = cnt;
+  __syncthreads();
+  int64_t base = out, total = 0;
+  for (int w = 0; w < NW; ++w) {
+    const int64_t c = part[w];
+    if (w < wp) base += c;
+    total += c;
+  }
+  for (int c0 = w0; c0 < w1; c0 += 32) {
+    const int wi = c0 + lane;
+    const uint32_t word = wi < w1 ? bits[wi] : 0u;
+    const int pc = __popc(word);
+    const int incl = warp_incl_scan(pc);
+    const int excl = incl - pc;
+    for (int j = 0; j < 32; ++j) {
+      const uint32_t wj = __shfl_sync(0xffffffffu, word, j);
+      if (!wj) continue;   // warp-uniform
+      const int oj = __shfl_sync(0xffffffffu, excl, j);
+      if ((wj >> lane) & 1u) {
+        const int64_t o = base + oj + __popc(wj & ((1u << lane) - 1u));
+        const uint32_t ci = (uint32_t)(c0 + j) * 32u + (uint32_t)lane;
+        C_col[o] = (int32_t)(wlo + ci);
+        C_val[o] = dvals[ci];
+      }
+    }
+    base += __shfl_sync(0xffffffffu, incl, 31);
+  }
+  __syncthreads();   // part[] is reused by the caller
+  return total;
 }
 
 // acquire a per-SM resume scratch slot (largest configuration: one CTA per SM)
@@ -701,15 +753,17 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
         res_next = res + p.resume_stride / 2;
         for (int64_t f = tid; f < nnzA; f += T) res[f] = 0;
       }
-      const int nwords = (int)((W + 31) / 32);
       int64_t out = PASS == 1 ? bm.cbase[0] : 0;
       int64_t total = 0;
       if (tid == 0 && PASS == 1 && p.n_dense_rows) atomicAdd(p.n_dense_rows, 1ull);
       for (int64_t w = 0; w < nwin; ++w) {
         const int64_t wlo = lo + w * W, whi = min(wlo + W, hi + 1);
+        // only the window's actual width is cleared and scanned (the last / only window of a
+        // row is usually much narrower than the scratchpad)
+        const int nwords = (int)((whi - wlo + 31) / 32);
         for (int i = tid; i < nwords; i += T) bits[i] = 0u;
         if (PASS == 1)
-          for (int64_t i = tid; i < W; i += T) dvals[i] = V(0);
+          for (int64_t i = tid; i < whi - wlo; i += T) dvals[i] = V(0);
         __syncthreads();
         // expand-balanced accumulation of the products falling into this window
         auto ins = [&](uint32_t col, V v, bool act) { dense_insert<PASS, V>(bits, dvals, (uint32_t)wlo, col, v, act); };
@@ -719,26 +773,19 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
         { int32_t* t_ = res; res = res_next; res_next = t_; }
         // ---- window epilogue: count (symbolic) / compact in column order (numeric) ----
         int64_t wtot = 0;
-        for (int base = 0; base < nwords; base += T) {
-          const int wi = base + tid;
-          const uint32_t word = wi < nwords ? bits[wi] : 0u;
-          const int64_t pc = __popc(word);
-          int64_t tot;
-          const int64_t pre = block_excl_scan<T>(pc, bm.scan_part, &tot);
-          if (PASS == 0 && chunks && word) atomicAdd(&chist[(wlo + (int64_t)wi * 32) >> p.chunk_shift], (int)pc);
-          if (PASS == 1 && word) {
-            uint32_t wd = word;
-            int64_t o = out + wtot + pre;
-            while (wd) {
-              const int b = __ffs(wd) - 1;
-              wd &= wd - 1;
-              const int64_t ci = (int64_t)wi * 32 + b;
-              p.C_col[o] = (int32_t)(wlo + ci);
-              p.C_val[o] = dvals[ci];
-              ++o;
-            }
+        if (PASS == 1) {
+          wtot = dense_emit<T, V>(bits, dvals, nwords, (uint32_t)wlo, out, p.C_col, p.C_val, bm.scan_part);
+        } else {
+          int cw = 0;
+          for (int wi = tid; wi < nwords; wi += T) {
+            const uint32_t word = bits[wi];
+            cw += __popc(word);
+            if (chunks && word) atomicAdd(&chist[(wlo + (int64_t)wi * 32) >> p.chunk_shift], __popc(word));
           }
-          wtot += tot;
+          cw = warp_sum(cw);
+          if (lane_id() == 0) bm.scan_part[warp_id()] = cw;
+          __syncthreads();
+          for (int w = 0; w < NW; ++w) wtot += bm.scan_part[w];
         }
         out += wtot;
         total += wtot;
