@@ -173,6 +173,7 @@ __global__ void __launch_bounds__(1024, 1) k_segments(SpgemmArgs<V> p, const Seg
     uint32_t* keys = reinterpret_cast<uint32_t*>(smem);
     V* vals = reinterpret_cast<V*>(smem + num_val_offset<V>(CFG));
     const uint32_t S = num_map_cap<V>(CFG);
+    const uint64_t mmult = mono_mult(range, S);
     for (uint32_t i = tid; i < S; i += T) { keys[i] = kEmptyKey; vals[i] = V(0); }
     if (tid == 0) s_wrap = 0;
     __syncthreads();
@@ -181,7 +182,7 @@ __global__ void __launch_bounds__(1024, 1) k_segments(SpgemmArgs<V> p, const Seg
         p, a0, alen, warp_id(), NW,
         [&](uint32_t col, V v, bool act) {
           uint32_t s = 0;
-          if (act) s = probe_insert_mono(keys, S, mono_slot(col, lo, range, S), col, &wrapped);
+          if (act) s = probe_insert_mono(keys, S, mono_slot(col, lo, mmult), col, &wrapped);
           bool leader;
           const V sum = warp_key_sum(col, v, leader);
           if (act && leader) atomicAdd(&vals[s], sum);

@@ -333,14 +333,19 @@ speck_status_t run_pass(speck_handle_t h, int pass, int lb, const int64_t* cat_s
                         const BinParams& bp, cudaStream_t s) {
   const int64_t m = a.m;
   if (!lb) {
-    // no load balancing: one configuration with room for R rows of the longest size
+    // no load balancing: one configuration with room for R rows of the longest size.
+    // Capacities are the maps' own (the long-row cap adjustment of the binned path does not
+    // apply: without balancing every row already fits below it).
+    BinParams own = bp;
+    for (int c = 0; c < kNumCfg; ++c)
+      own.cap[c] = pass == 0 ? (int64_t)sym_map_fill(c) : (int64_t)num_map_fill<V>(c);
     int cfg = -1, R = 1;
     for (int c = 0; c < kNumCfg; ++c)
-      if (need_max * kMaxGroupRows <= bp.cap[c]) { cfg = c; R = kMaxGroupRows; break; }
+      if (need_max * kMaxGroupRows <= own.cap[c]) { cfg = c; R = kMaxGroupRows; break; }
     if (cfg < 0) {
-      cfg = cfg_for(bp, need_max);
+      cfg = cfg_for(own, need_max);
       if (cfg >= kNumCfg) cfg = kNumCfg - 1;
-      R = (int)std::max<int64_t>(1, std::min<int64_t>(kMaxGroupRows, bp.cap[cfg] / std::max<int64_t>(need_max, 1)));
+      R = (int)std::max<int64_t>(1, std::min<int64_t>(kMaxGroupRows, own.cap[cfg] / std::max<int64_t>(need_max, 1)));
     }
     a.rows = nullptr;
     a.n_entries = m;

@@ -36,7 +36,6 @@ struct BlockMeta {
   int32_t cseg[kMaxGroupRows + 1];   // numeric: prefix of cnt_r over the block
   uint32_t rbase[kMaxGroupRows + 1]; // hash region start of each row
   int32_t rcnt[kMaxGroupRows];       // symbolic: distinct columns per row
-  int32_t rg[kMaxGroupRows];         // warp-per-row path: group size per row
   int32_t rlo[kMaxGroupRows];        // colmin / colmax per row (order-preserving hash)
   int32_t rhi[kMaxGroupRows];
   int32_t rwrap[kMaxGroupRows];      // block path: a probing run of the row wrapped around
@@ -80,9 +79,14 @@ __device__ __forceinline__ uint32_t probe_insert(uint32_t* keys, uint32_t S, uin
 // runs.  With linear probing and no wrap-around, every key sits in the run ("cluster") that
 // contains its home, and clusters appear in column order; an entry's position in the sorted
 // row is therefore (#occupied slots before its cluster) + (rank of its key inside the cluster).
-__device__ __forceinline__ uint32_t mono_slot(uint32_t col, uint32_t lo, uint32_t range, uint32_t S) {
-  const uint32_t sh = S - (S >> 3);
-  return (uint32_t)(((uint64_t)(col - lo) * sh) / range);
+// home = floor((col - lo) * mult / 2^32) with mult = floor(sh * 2^32 / range), sh = 7/8 S:
+// monotone in col, < sh, and a multiply per product instead of a 64-bit division.
+__device__ __forceinline__ uint64_t mono_mult(uint32_t range, uint32_t S) {
+  const uint64_t sh = S - (S >> 3);
+  return range ? (sh << 32) / range : 0;
+}
+__device__ __forceinline__ uint32_t mono_slot(uint32_t col, uint32_t lo, uint64_t mult) {
+  return (uint32_t)(((uint64_t)(col - lo) * mult) >> 32);
 }
 
 // linear probing that reports a wrap-around (which breaks the cluster order)
@@ -109,6 +113,46 @@ __device__ __forceinline__ int cluster_position(const uint32_t* keys, uint32_t S
     rank += k < key;
   }
   return before - (int)(s - cs) + rank;
+}
+
+// Sorted write-out of the slots [c0, c0+32) of an ordered map region (all 32 lanes call it;
+// `before` = occupied slots before c0, advanced on return).  Probing runs that lie inside the
+// chunk are ranked with shuffles — position = (occupied before me) + (#later run members with a
+// smaller key) - (#earlier members with a larger key) — in max-run-length steps without
+// divergence; only runs crossing a chunk edge walk the map (cluster_position).
+template <typename V>
+__device__ __forceinline__ void ordered_chunk_emit(const uint32_t* rk, const V* rv, uint32_t S, uint32_t c0, int& before,
+                                                   int64_t ob, int32_t* __restrict__ C_col, V* __restrict__ C_val) {
+  const int lane = lane_id();
+  const uint32_t s = c0 + lane;
+  const uint32_t kk = s < S ? rk[s] : kEmptyKey;
+  const bool occ_me = kk != kEmptyKey;
+  const uint32_t occ = __ballot_sync(0xffffffffu, occ_me);
+  const bool prev_occ = c0 > 0 && rk[c0 - 1] != kEmptyKey;          // same address on all lanes
+  const bool next_occ = c0 + 32 < S && rk[c0 + 32] != kEmptyKey;
+  const uint32_t starts = occ & ~((occ << 1) | (prev_occ ? 1u : 0u));
+  const uint32_t ends = occ & ~((occ >> 1) | (next_occ ? 0x80000000u : 0u));
+  const uint32_t lt = (1u << lane) - 1u;
+  const uint32_t ms = starts & (lt | (1u << lane));
+  const int cs = ms ? 31 - __clz(ms) : -1;      // -1: the run began before this chunk
+  const uint32_t me = ends & ~lt;
+  const int ce = me ? __ffs(me) - 1 : 32;       // 32: the run continues after it
+  const bool inside = occ_me && cs >= 0 && ce < 32;
+  const int L = (int)__reduce_max_sync(0xffffffffu, inside ? (unsigned)(ce - cs) : 0u);
+  int after_smaller = 0, before_larger = 0;
+  for (int d = 1; d <= L; ++d) {
+    const uint32_t kd = __shfl_down_sync(0xffffffffu, kk, d);
+    const uint32_t ku = __shfl_up_sync(0xffffffffu, kk, d);
+    after_smaller += (lane + d <= ce && kd < kk);
+    before_larger += (lane - d >= cs && ku > kk);
+  }
+  if (occ_me) {
+    const int mypre = before + __popc(occ & lt);
+    const int o = inside ? mypre + after_smaller - before_larger : cluster_position(rk, S, s, kk, mypre);
+    C_col[ob + o] = (int32_t)kk;
+    C_val[ob + o] = rv[s];
+  }
+  before += __popc(occ);
 }
 
 // symbolic insert: true if the key was new
@@ -187,17 +231,8 @@ __device__ void block_write_ordered(const uint32_t* rk, const V* rv, uint32_t S,
   __syncthreads();
   int before = 0;
   for (int w = 0; w < wp; ++w) before += (int)part[w];
-  for (uint32_t c0 = w0; c0 < w1; c0 += 32) {
-    const uint32_t s = c0 + lane;
-    const uint32_t kk = s < w1 ? rk[s] : kEmptyKey;
-    const uint32_t occ = __ballot_sync(0xffffffffu, kk != kEmptyKey);
-    if (kk != kEmptyKey) {
-      const int o = cluster_position(rk, S, s, kk, before + __popc(occ & ((1u << lane) - 1u)));
-      C_col[ob + o] = (int32_t)kk;
-      C_val[ob + o] = rv[s];
-    }
-    before += __popc(occ);
-  }
+  // warp ranges are 32-slot aligned and w1 is a chunk boundary or S, so chunks never straddle
+  for (uint32_t c0 = w0; c0 < w1; c0 += 32) ordered_chunk_emit<V>(rk, rv, S, c0, before, ob, C_col, C_val);
   __syncthreads();
 }
 
@@ -477,8 +512,6 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
         bm.rlo[l] = cmn;
         bm.rhi[l] = cmx;
         bm.rwrap[l] = 0;
-        // per-row group size for the warp-per-row path (local LB with T = one warp)
-        bm.rg[l] = p.fixed_g > 0 ? min(p.fixed_g, 32) : local_group_size(32, alen, pr, ml);
       }
       if (l == 0) {
         bm.aoff[0] = 0; bm.cseg[0] = 0; bm.rbase[0] = 0;
@@ -541,7 +574,7 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
         const int64_t a0 = bm.astart[r];
         const int alen = (int)(bm.aoff[r + 1] - bm.aoff[r]);
         const uint32_t mlo = (uint32_t)bm.rlo[r];
-        const uint32_t mrange = (uint32_t)(bm.rhi[r] - bm.rlo[r] + 1);
+        const uint64_t mmult = mono_mult((uint32_t)(bm.rhi[r] - bm.rlo[r] + 1), S);
         // long rows use the order-preserving map (sorted write-out without a sort network);
         // short rows keep the scrambled hash (robust to clustered columns) and rank counting
         const bool ordered = PASS == 1 && bm.cseg[r + 1] - bm.cseg[r] > kSmallSeg;
@@ -550,13 +583,19 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
           if (PASS == 0) {
             if (act) newc += hash_insert_key(rk, S, col);
           } else {
+            const uint32_t peers = __match_any_sync(0xffffffffu, col);
+            const uint32_t lt = (1u << lane_id()) - 1u;
             uint32_t s = 0;
-            if (act)
-              s = probe_insert_mono(rk, S, ordered ? mono_slot(col, mlo, mrange, S) : hash_slot(col, S), col, &wrapped);
-            bool leader;
-            const V sum = warp_key_sum(col, v, leader);
-            if (act && leader) rv[s] += sum;   // the region is private to this warp: no atomic
-            __syncwarp();
+            if (act && !(peers & lt))
+              s = probe_insert_mono(rk, S, ordered ? mono_slot(col, mlo, mmult) : hash_slot(col, S), col, &wrapped);
+            s = __shfl_sync(0xffffffffu, s, __ffs(peers) - 1);   // the key's slot, from its first lane
+            // the region is private to this warp: equal keys add in rounds, no atomics
+            const int rank = __popc(peers & lt);
+            const int maxg = (int)__reduce_max_sync(0xffffffffu, (unsigned)__popc(peers));
+            for (int t = 0; t < maxg; ++t) {
+              if (act && rank == t) rv[s] += v;
+              __syncwarp();
+            }
           }
         });
         if (PASS == 0) {
@@ -567,17 +606,7 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
           // the cluster) — the row comes out sorted without moving anything in shared memory
           const int64_t ob = bm.cbase[r];
           int before = 0;
-          for (uint32_t c0 = 0; c0 < S; c0 += 32) {
-            const uint32_t s = c0 + lane;
-            const uint32_t kk = s < S ? rk[s] : kEmptyKey;
-            const uint32_t occ = __ballot_sync(0xffffffffu, kk != kEmptyKey);
-            if (kk != kEmptyKey) {
-              const int o = cluster_position(rk, S, s, kk, before + __popc(occ & ((1u << lane) - 1u)));
-              p.C_col[ob + o] = (int32_t)kk;
-              p.C_val[ob + o] = rv[s];
-            }
-            before += __popc(occ);
-          }
+          for (uint32_t c0 = 0; c0 < S; c0 += 32) ordered_chunk_emit<V>(rk, rv, S, c0, before, ob, p.C_col, p.C_val);
         } else {
           // a probing run wrapped around: compact the region in place, then sort and write
           int pos = 0;
@@ -637,7 +666,8 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
         const uint32_t rb = bm.rbase[r], S = bm.rbase[r + 1] - rb;
         uint32_t* rk = keys + rb;
         V* rv = vals + rb;
-        const uint32_t mlo = (uint32_t)bm.rlo[r], mrange = (uint32_t)(bm.rhi[r] - bm.rlo[r] + 1);
+        const uint32_t mlo = (uint32_t)bm.rlo[r];
+        const uint64_t mmult = mono_mult((uint32_t)(bm.rhi[r] - bm.rlo[r] + 1), S);
         const bool ordered = bm.ordered;
         int newc = 0, wrapped = 0;
         expand_row<PASS, V>(p, bm.astart[r], (int)(bm.aoff[r + 1] - bm.aoff[r]), warp_id(), NW,
@@ -647,7 +677,7 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
                               } else {
                                 uint32_t s = 0;
                                 if (act)
-                                  s = probe_insert_mono(rk, S, ordered ? mono_slot(col, mlo, mrange, S) : hash_slot(col, S),
+                                  s = probe_insert_mono(rk, S, ordered ? mono_slot(col, mlo, mmult) : hash_slot(col, S),
                                                         col, &wrapped);
                                 bool leader;
                                 const V sum = warp_key_sum(col, v, leader);

@@ -48,8 +48,11 @@ def main(rep, launch=0):
                 pass
     ts = sum(o[0] for o in out) or 1
     ti = sum(o[1] for o in out) or 1
-    print(f"top source lines (stall samples {ts}, warp instructions {ti}):")
+    print(f"top source lines by stall samples (total {ts}; warp instructions {ti}):")
     for o in sorted(out, reverse=True)[:20]:
+        print(f"  {100 * o[0] / ts:5.1f}% stalls {100 * o[1] / ti:5.1f}% inst  {o[2]}:{o[3]}  {o[4]}")
+    print("top source lines by executed warp instructions:")
+    for o in sorted(out, key=lambda x: -x[1])[:15]:
         print(f"  {100 * o[0] / ts:5.1f}% stalls {100 * o[1] / ti:5.1f}% inst  {o[2]}:{o[3]}  {o[4]}")
 
 
