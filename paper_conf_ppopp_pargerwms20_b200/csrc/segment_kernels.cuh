@@ -57,7 +57,8 @@ struct SegPlanArgs {
   const int32_t* chunk_cnt;
   int nchunks;
   int shift;
-  int64_t limit;           // numeric long-row threshold = entries of a hashed segment
+  int64_t limit;           // numeric long-row threshold (entries of the largest map)
+  int64_t seg_limit;       // max entries of a hashed segment (map of kSegCfg)
   int64_t dense_window;    // columns of one dense window of the largest configuration
   int64_t map_slots;       // slots of the largest numeric hash map
   int prefer_parallel;     // few long rows: always split (parallelism across SMs)
@@ -76,7 +77,7 @@ __device__ __forceinline__ bool use_windows(const SegPlanArgs& a, int32_t row, i
   const int64_t avg = dA > 0 ? a.prods[row] / dA + 1 : 1;
   int64_t lg = 1;
   while ((int64_t)1 << lg < avg) ++lg;
-  const int64_t nseg = cnt / a.limit + 1;
+  const int64_t nseg = cnt / a.seg_limit + 1;
   const int64_t win_cost = nwin * (a.dense_window / 8 + dA * (1 + lg));
   const int64_t seg_cost = nseg * (dA * 2 * lg + map_slots / 4);
   return win_cost <= seg_cost;
@@ -93,7 +94,7 @@ __global__ void k_seg_count(SegPlanArgs a, int64_t* __restrict__ nseg) {
     if (use_windows(a, row, cnt, a.map_slots)) {
       n = 1;
     } else {
-      plan_row_segments(a.chunk_cnt + e * a.nchunks, a.colmin[row] >> a.shift, a.colmax[row] >> a.shift, a.limit,
+      plan_row_segments(a.chunk_cnt + e * a.nchunks, a.colmin[row] >> a.shift, a.colmax[row] >> a.shift, a.seg_limit,
                         [&](int, int, int64_t, int64_t, bool) { ++n; });
     }
   }
@@ -118,7 +119,7 @@ __global__ void k_seg_emit(SegPlanArgs a, const int64_t* __restrict__ seg_off, S
     return;
   }
   const int shift = a.shift;
-  plan_row_segments(a.chunk_cnt + e * a.nchunks, lo >> shift, hi >> shift, a.limit,
+  plan_row_segments(a.chunk_cnt + e * a.nchunks, lo >> shift, hi >> shift, a.seg_limit,
                     [&](int ca, int cb, int64_t n, int64_t done, bool dense) {
                       Seg s;
                       s.row = row;
@@ -156,8 +157,9 @@ __device__ int64_t dense_window_pass(const SpgemmArgs<V>& p, int64_t a0, int ale
 
 // One CTA (the largest configuration, 1 CTA/SM) per job.
 template <typename V>
-__global__ void __launch_bounds__(1024, 1) k_segments(SpgemmArgs<V> p, const Seg* __restrict__ segs) {
-  constexpr int CFG = kNumCfg - 1;
+__global__ void __launch_bounds__(kCfgThreads[kSegCfg], 1024 / kCfgThreads[kSegCfg])
+    k_segments(SpgemmArgs<V> p, const Seg* __restrict__ segs) {
+  constexpr int CFG = kSegCfg;
   constexpr int T = kCfgThreads[CFG];
   constexpr int NW = T / 32;
   extern __shared__ __align__(16) unsigned char smem[];
@@ -220,16 +222,13 @@ __global__ void __launch_bounds__(1024, 1) k_segments(SpgemmArgs<V> p, const Seg
     if (sg.dense == SEG_DENSE) {
       dense_window_pass<V, T>(p, a0, alen, bits, dvals, lo, hi, sg.out, part, SegRange{p.B_col, lo, hi});
     } else {
-      // whole row, windows in ascending column order with resume positions
-      int32_t* res = p.resume + (int64_t)smid() * p.resume_stride;   // 1 CTA per SM: private slot
-      int32_t* res_next = res + p.resume_stride / 2;
-      for (int f = tid; f < alen; f += T) res[f] = 0;
+      // whole row, dense windows in ascending column order; each referenced B
+      // row is located in the window by binary search (two CTAs share an SM, so the per-SM
+      // resume slots of the largest configuration are not used here)
       int64_t out = sg.out;
       for (uint32_t wlo = lo; wlo < hi; wlo = (uint32_t)min((int64_t)hi, (int64_t)wlo + W)) {
         const uint32_t whi = (uint32_t)min((int64_t)hi, (int64_t)wlo + W);
-        out += dense_window_pass<V, T>(p, a0, alen, bits, dvals, wlo, whi, out, part,
-                                       WindowRange{res, res_next, p.B_col, whi});
-        int32_t* t_ = res; res = res_next; res_next = t_;   // dense_window_pass ends with a barrier
+        out += dense_window_pass<V, T>(p, a0, alen, bits, dvals, wlo, whi, out, part, SegRange{p.B_col, wlo, whi});
       }
     }
   }

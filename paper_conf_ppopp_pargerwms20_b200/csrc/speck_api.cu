@@ -203,7 +203,7 @@ speck_status_t set_smem_attrs(speck_handle_t h) {
   for (int c = 0; c < kNumCfg; ++c)
     for (int pass = 0; pass < 2; ++pass)
       CK(cudaFuncSetAttribute(spgemm_fn<V>(c, pass), cudaFuncAttributeMaxDynamicSharedMemorySize, kCfgMapBytes[c]));
-  CK(cudaFuncSetAttribute(k_segments<V>, cudaFuncAttributeMaxDynamicSharedMemorySize, kCfgMapBytes[kNumCfg - 1]));
+  CK(cudaFuncSetAttribute(k_segments<V>, cudaFuncAttributeMaxDynamicSharedMemorySize, kCfgMapBytes[kSegCfg]));
   return SPECK_OK;
 }
 
@@ -260,7 +260,7 @@ template <typename V>
 void plan_segments(speck_handle_t h, int64_t ncols) {
   h->long_thr = num_map_fill<V>(kNumCfg - 1);
   int s = 0;
-  while ((int64_t)1 << (s + 1) <= num_dense_window<V>(kNumCfg - 1)) ++s;
+  while ((int64_t)1 << (s + 1) <= num_dense_window<V>(kSegCfg)) ++s;
   h->seg_shift = s;
   h->nchunks = (int)((ncols + ((int64_t)1 << s) - 1) >> s);
   h->seg_enabled = h->opt_force_acc != 2 && h->opt_segments != 0 && h->nchunks >= 1 && h->nchunks <= kMaxChunks;
@@ -319,8 +319,9 @@ SegPlanArgs seg_plan_args(speck_handle_t h, const int64_t* C_rp) {
   s.nchunks = h->nchunks;
   s.shift = h->seg_shift;
   s.limit = h->long_thr;
-  s.dense_window = num_dense_window<V>(kNumCfg - 1);
-  s.map_slots = num_map_cap<V>(kNumCfg - 1);
+  s.dense_window = num_dense_window<V>(kSegCfg);
+  s.map_slots = num_map_cap<V>(kSegCfg);
+  s.seg_limit = num_map_fill<V>(kSegCfg);
   // few candidates: split every long row so its work spreads over the SMs
   s.prefer_parallel = h->n_cand < 4 * (int64_t)h->num_sms ? 1 : 0;
   return s;
@@ -369,7 +370,7 @@ speck_status_t run_pass(speck_handle_t h, int pass, int lb, const int64_t* cat_s
   int si = 0;
   const int32_t* bins = static_cast<const int32_t*>(h->bins.p);
   if (segs) {
-    k_segments<V><<<(unsigned)h->n_segs, kCfgThreads[kNumCfg - 1], kCfgMapBytes[kNumCfg - 1], h->streams[si]>>>(
+    k_segments<V><<<(unsigned)h->n_segs, kCfgThreads[kSegCfg], kCfgMapBytes[kSegCfg], h->streams[si]>>>(
         a, static_cast<const Seg*>(h->segs.p));
     CKL();
     si = (si + 1) % ns;

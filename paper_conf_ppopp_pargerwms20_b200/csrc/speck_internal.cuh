@@ -50,6 +50,9 @@ enum Cat : int {
 // columns (2^s <= one dense window of the largest configuration: s = 15 fp32, 14 fp64), at
 // most kMaxChunks per row.
 constexpr int kMaxChunks = 1024;
+// Long-row jobs run in configuration 3 (512 threads, 2 CTAs per SM), so one CTA's barriers
+// overlap with the other's work; segments hold up to that map's fill.
+constexpr int kSegCfg = kNumCfg - 2;
 struct Seg {
   int32_t row;
   int32_t col_lo;   // first column of the segment

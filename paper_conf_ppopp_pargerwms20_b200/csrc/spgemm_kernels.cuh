@@ -6,17 +6,18 @@
 // block merge of Alg. 2 (merged small-row bin only), and for each block:
 //   1. picks the accumulator: hash map, dense array; direct
 //      rows have their own kernel below;
-//   2. picks the local-load-balancer group size g and lets k = T/g groups of
-//      g threads stream the referenced rows of B (coalesced within a group);
+//   2. enumerates the products with the expand-balanced local load balancer (expand_row:
+//      the B200 form of P:867-970 — every lane gets the same number of products);
 //   3. symbolic: counts the distinct columns per row;
-//      numeric: accumulates values, then compacts and SORTS each row in shared memory
-//      before writing it at its C row offset.
+//      numeric: accumulates values and writes each row SORTED at its C row offset
+//      (P:1121-1148).
 //
-// B200 differences from the paper's Titan V design (DESIGN.md §Kernels):
+// B200 differences from the paper's Titan V design (DESIGN.md §5):
 //   * merged rows use per-row regions of the map instead of a 5-bit row + 27-bit column
 //     compound key, so blocks of up to 32 rows work for any column count;
-//   * every hash row is sorted in shared memory (rank counting for short rows, a bitonic
-//     network for long ones) — 227 KB per CTA makes a global radix-sort pass unnecessary;
+//   * multi-row blocks run one warp per row (no block barriers, warp-aggregated updates);
+//   * rows > 64 entries use an order-preserving hash: runs are insertion-sorted in place and
+//     the write-out is a compaction; short rows use rank counting; no global sort pass;
 //   * dense windows of rows needing several windows keep resume positions per referenced
 //     B row in a per-SM global scratch slot.
 #pragma once
@@ -102,57 +103,30 @@ __device__ __forceinline__ uint32_t probe_insert_mono(uint32_t* keys, uint32_t S
   }
 }
 
-// Position of the occupied slot s inside its row: `before` = occupied slots before s.
-__device__ __forceinline__ int cluster_position(const uint32_t* keys, uint32_t S, uint32_t s, uint32_t key, int before) {
-  uint32_t cs = s;
-  while (cs > 0 && keys[cs - 1] != kEmptyKey) --cs;
-  int rank = 0;
-  for (uint32_t t = cs; t < S; ++t) {
-    const uint32_t k = keys[t];
-    if (k == kEmptyKey) break;
-    rank += k < key;
-  }
-  return before - (int)(s - cs) + rank;
-}
-
-// Sorted write-out of the slots [c0, c0+32) of an ordered map region (all 32 lanes call it;
-// `before` = occupied slots before c0, advanced on return).  Probing runs that lie inside the
-// chunk are ranked with shuffles — position = (occupied before me) + (#later run members with a
-// smaller key) - (#earlier members with a larger key) — in max-run-length steps without
-// divergence; only runs crossing a chunk edge walk the map (cluster_position).
+// Sort every probing run of an ordered map region in place (keys and values): the thread
+// owning a run's first slot walks the run and insertion-sorts it (runs are short and nearly
+// sorted).  Threads t0, t0+step, ... examine the slots.  After this (and a barrier), the
+// occupied slots are in column order, so the write-out is a plain order-preserving compaction.
 template <typename V>
-__device__ __forceinline__ void ordered_chunk_emit(const uint32_t* rk, const V* rv, uint32_t S, uint32_t c0, int& before,
-                                                   int64_t ob, int32_t* __restrict__ C_col, V* __restrict__ C_val) {
-  const int lane = lane_id();
-  const uint32_t s = c0 + lane;
-  const uint32_t kk = s < S ? rk[s] : kEmptyKey;
-  const bool occ_me = kk != kEmptyKey;
-  const uint32_t occ = __ballot_sync(0xffffffffu, occ_me);
-  const bool prev_occ = c0 > 0 && rk[c0 - 1] != kEmptyKey;          // same address on all lanes
-  const bool next_occ = c0 + 32 < S && rk[c0 + 32] != kEmptyKey;
-  const uint32_t starts = occ & ~((occ << 1) | (prev_occ ? 1u : 0u));
-  const uint32_t ends = occ & ~((occ >> 1) | (next_occ ? 0x80000000u : 0u));
-  const uint32_t lt = (1u << lane) - 1u;
-  const uint32_t ms = starts & (lt | (1u << lane));
-  const int cs = ms ? 31 - __clz(ms) : -1;      // -1: the run began before this chunk
-  const uint32_t me = ends & ~lt;
-  const int ce = me ? __ffs(me) - 1 : 32;       // 32: the run continues after it
-  const bool inside = occ_me && cs >= 0 && ce < 32;
-  const int L = (int)__reduce_max_sync(0xffffffffu, inside ? (unsigned)(ce - cs) : 0u);
-  int after_smaller = 0, before_larger = 0;
-  for (int d = 1; d <= L; ++d) {
-    const uint32_t kd = __shfl_down_sync(0xffffffffu, kk, d);
-    const uint32_t ku = __shfl_up_sync(0xffffffffu, kk, d);
-    after_smaller += (lane + d <= ce && kd < kk);
-    before_larger += (lane - d >= cs && ku > kk);
+__device__ __forceinline__ void sort_runs(uint32_t* keys, V* vals, uint32_t S, uint32_t t0, uint32_t step) {
+  for (uint32_t s = t0; s < S; s += step) {
+    if (keys[s] == kEmptyKey || (s > 0 && keys[s - 1] != kEmptyKey)) continue;   // not a run start
+    uint32_t e = s + 1;
+    while (e < S && keys[e] != kEmptyKey) ++e;
+    for (uint32_t i = s + 1; i < e; ++i) {
+      const uint32_t k = keys[i];
+      if (keys[i - 1] <= k) continue;
+      const V v = vals[i];
+      uint32_t j = i;
+      while (j > s && keys[j - 1] > k) {
+        keys[j] = keys[j - 1];
+        vals[j] = vals[j - 1];
+        --j;
+      }
+      keys[j] = k;
+      vals[j] = v;
+    }
   }
-  if (occ_me) {
-    const int mypre = before + __popc(occ & lt);
-    const int o = inside ? mypre + after_smaller - before_larger : cluster_position(rk, S, s, kk, mypre);
-    C_col[ob + o] = (int32_t)kk;
-    C_val[ob + o] = rv[s];
-  }
-  before += __popc(occ);
 }
 
 // symbolic insert: true if the key was new
@@ -162,20 +136,12 @@ __device__ __forceinline__ bool hash_insert_key(uint32_t* keys, uint32_t S, uint
   return is_new;
 }
 
-// numeric insert-or-accumulate
-template <typename V>
-__device__ __forceinline__ void hash_accumulate(uint32_t* keys, V* vals, uint32_t S, uint32_t col, V v) {
-  bool is_new;
-  const uint32_t s = probe_insert(keys, S, hash_slot(col, S), col, &is_new);
-  atomicAdd(&vals[s], v);
-}
-
 // Bitonic sort of (keys, vals)[0, n) ascending in shared memory, any n: the "flip"
 // formulation keeps all sub-sorts ascending, so comparisons with a partner index >= n
 // (a virtual +inf) are no-ops and can be skipped.
 // WARP = true: one warp sorts (lanes 0..31, __syncwarp between stages).
 template <int T, typename V, bool WARP = false>
-__device__ void smem_bitonic_sort(uint32_t* keys, V* vals, int n) {
+__device__ __noinline__ void smem_bitonic_sort(uint32_t* keys, V* vals, int n) {
   if (n <= 1) return;
   const int t0 = WARP ? (int)(threadIdx.x & 31) : (int)threadIdx.x;
   int P = 1;
@@ -212,16 +178,18 @@ __device__ void smem_bitonic_sort(uint32_t* keys, V* vals, int n) {
   }
 }
 
-// Block-wide write-out of one ordered map region [0, S): warp-contiguous slot ranges, one
-// block scan of the per-warp occupancy, then every entry goes to its sorted position.
-// Contains two block barriers; `part` = >= 32 int64 of shared scratch.
+// Block-wide write-out of one ordered map region [0, S): sort the probing runs in place,
+// then an order-preserving compaction — warp-contiguous slot ranges, one block-level prefix
+// of the per-warp occupancy, coalesced writes.  Barriers inside; `part` = >= 32 int64 scratch.
 template <int T, typename V>
-__device__ void block_write_ordered(const uint32_t* rk, const V* rv, uint32_t S, int64_t ob, int32_t* __restrict__ C_col,
+__device__ void block_write_ordered(uint32_t* rk, V* rv, uint32_t S, int64_t ob, int32_t* __restrict__ C_col,
                                     V* __restrict__ C_val, int64_t* part) {
   constexpr int NW = T / 32;
   const int lane = lane_id(), wp = warp_id();
+  sort_runs<V>(rk, rv, S, threadIdx.x, T);
   const uint32_t SW = ((S + NW - 1) / NW + 31u) & ~31u;
   const uint32_t w0 = min(S, wp * SW), w1 = min(S, w0 + SW);
+  __syncthreads();
   int cw = 0;
   for (uint32_t c0 = w0; c0 < w1; c0 += 32) {
     const uint32_t s = c0 + lane;
@@ -231,8 +199,17 @@ __device__ void block_write_ordered(const uint32_t* rk, const V* rv, uint32_t S,
   __syncthreads();
   int before = 0;
   for (int w = 0; w < wp; ++w) before += (int)part[w];
-  // warp ranges are 32-slot aligned and w1 is a chunk boundary or S, so chunks never straddle
-  for (uint32_t c0 = w0; c0 < w1; c0 += 32) ordered_chunk_emit<V>(rk, rv, S, c0, before, ob, C_col, C_val);
+  for (uint32_t c0 = w0; c0 < w1; c0 += 32) {
+    const uint32_t s = c0 + lane;
+    const uint32_t kk = s < w1 ? rk[s] : kEmptyKey;
+    const uint32_t occ = __ballot_sync(0xffffffffu, kk != kEmptyKey);
+    if (kk != kEmptyKey) {
+      const int64_t o = ob + before + __popc(occ & ((1u << lane) - 1u));
+      C_col[o] = (int32_t)kk;
+      C_val[o] = rv[s];
+    }
+    before += __popc(occ);
+  }
   __syncthreads();
 }
 
@@ -300,16 +277,16 @@ __device__ __forceinline__ void expand_row(const SpgemmArgs<V>& p, int64_t a0, i
     const int incl = warp_incl_scan(blen);
     const int excl = incl - blen;
     const int Pb = __shfl_sync(0xffffffffu, incl, 31);
-    for (int p0 = c_first * CH; p0 < Pb; p0 += c_step * CH) {
-      uint32_t col[kPPL];
-      V v[kPPL];
+    // locate the products of chunk q0 and issue their loads (not consumed here)
+    auto gather = [&](int q0, uint32_t (&c)[kPPL], V (&bv)[kPPL], int (&ow)[kPPL]) {
 #pragma unroll
       for (int i = 0; i < kPPL; ++i) {
-        col[i] = 0x80000000u | (uint32_t)lane;
-        v[i] = V(0);
-        if (p0 + 32 * i >= Pb) continue;   // warp-uniform: the whole sub-chunk is past the row
-        const int pp = p0 + lane + 32 * i;
-        int lo = 0;   // owner lane: smallest o with incl_o > pp
+        c[i] = 0x80000000u | (uint32_t)lane;   // inactive lanes keep a key that is never a real column
+        bv[i] = V(0);
+        ow[i] = 0;
+        if (q0 + 32 * i >= Pb) continue;       // warp-uniform: the whole sub-chunk is past the row
+        const int pp = q0 + lane + 32 * i;
+        int lo = 0;                            // owner lane: smallest o with incl_o > pp
 #pragma unroll
         for (int step = 16; step > 0; step >>= 1) {
           const int probe = __shfl_sync(0xffffffffu, incl, lo + step - 1);
@@ -317,15 +294,25 @@ __device__ __forceinline__ void expand_row(const SpgemmArgs<V>& p, int64_t a0, i
         }
         const int o = lo > 31 ? 31 : lo;
         const int64_t idx = __shfl_sync(0xffffffffu, bst, o) + (pp - __shfl_sync(0xffffffffu, excl, o));
-        const V ao = PASS == 1 ? __shfl_sync(0xffffffffu, a, o) : V(0);
-        if (pp < Pb) {   // inactive lanes keep a key that is never a real column (< 2^31)
-          col[i] = (uint32_t)p.B_col[idx];
-          if (PASS == 1) v[i] = ao * ldv(p.B_val + idx);
+        ow[i] = o;
+        if (pp < Pb) {
+          c[i] = (uint32_t)p.B_col[idx];
+          if (PASS == 1) bv[i] = ldv(p.B_val + idx);
         }
       }
+    };
+    // gather a chunk (kPPL independent loads per lane), then insert it
+    uint32_t ca[kPPL];
+    V va[kPPL];
+    int oa[kPPL];
+    for (int p0 = c_first * CH; p0 < Pb; p0 += c_step * CH) {
+      gather(p0, ca, va, oa);
 #pragma unroll
-      for (int i = 0; i < kPPL; ++i)
-        if (p0 + 32 * i < Pb) ins(col[i], v[i], p0 + lane + 32 * i < Pb);   // uniform skip of empty sub-chunks
+      for (int i = 0; i < kPPL; ++i) {
+        if (p0 + 32 * i >= Pb) continue;   // uniform skip of empty sub-chunks
+        const V ao = PASS == 1 ? __shfl_sync(0xffffffffu, a, oa[i]) : V(0);
+        ins(ca[i], ao * va[i], p0 + lane + 32 * i < Pb);
+      }
     }
   }
 }
@@ -432,6 +419,100 @@ __device__ __forceinline__ unsigned smid() {
   asm volatile("mov.u32 %0, %%smid;" : "=r"(r));
   return r;
 }
+
+// Warp-path write-out of a scrambled (or wrapped) map region: compact in place, then rank
+// counting for <= kSmallSeg entries or a warp bitonic sort.  Out of line.
+template <typename V>
+__device__ __noinline__ void warp_row_sorted_write(uint32_t* rk, V* rv, uint32_t S, int64_t ob, int32_t* __restrict__ C_col,
+                                                   V* __restrict__ C_val) {
+  const int lane = lane_id();
+  int pos = 0;
+  for (uint32_t c0 = 0; c0 < S; c0 += 32) {
+    const uint32_t s = c0 + lane;
+    uint32_t kk = kEmptyKey;
+    V vv = V(0);
+    if (s < S) { kk = rk[s]; vv = rv[s]; }
+    const uint32_t occ = __ballot_sync(0xffffffffu, kk != kEmptyKey);
+    __syncwarp();
+    if (kk != kEmptyKey) {
+      const int o = pos + __popc(occ & ((1u << lane) - 1u));
+      rk[o] = kk;
+      rv[o] = vv;
+    }
+    pos += __popc(occ);
+    __syncwarp();
+  }
+  const int cnt = pos;
+  if (cnt <= kSmallSeg) {
+    // all lanes read key j together (shared-memory broadcast)
+    for (int e0 = 0; e0 < cnt; e0 += 32) {
+      const int e = e0 + lane;
+      const uint32_t key = e < cnt ? rk[e] : 0xffffffffu;
+      const V val = e < cnt ? rv[e] : V(0);
+      int rank = 0;
+      for (int j = 0; j < cnt; ++j) rank += rk[j] < key;
+      if (e < cnt) {
+        C_col[ob + rank] = (int32_t)key;
+        C_val[ob + rank] = val;
+      }
+    }
+  } else {
+    smem_bitonic_sort<32, V, true>(rk, rv, cnt);
+    for (int e = lane; e < cnt; e += 32) {
+      C_col[ob + e] = (int32_t)rk[e];
+      C_val[ob + e] = rv[e];
+    }
+  }
+}
+
+// Block-path write-out of scrambled (or wrapped) maps: order-preserving compaction of all row
+// regions, rank counting for short rows, bitonic sort for long ones.  Out of line.
+template <int T, typename V>
+__device__ __noinline__ void block_sorted_write(uint32_t* keys, V* vals, uint32_t capt, BlockMeta& bm,
+                                                int32_t* __restrict__ C_col, V* __restrict__ C_val) {
+  const int tid = threadIdx.x;
+  const int nr = bm.nr;
+  int64_t running = 0;
+  for (uint32_t base = 0; base < capt; base += T) {
+    const uint32_t s = base + tid;
+    uint32_t kk = kEmptyKey;
+    V vv = V(0);
+    if (s < capt) { kk = keys[s]; vv = vals[s]; }
+    const int64_t fl = kk != kEmptyKey;
+    int64_t tot;
+    const int64_t pos = block_excl_scan<T>(fl, bm.scan_part, &tot);
+    if (fl) { keys[running + pos] = kk; vals[running + pos] = vv; }
+    running += tot;
+    __syncthreads();
+  }
+  const int ncnt = (int)bm.cnt;
+  int rr = 0;
+  for (int i = tid; i < ncnt; i += T) {
+    while (i >= bm.cseg[rr + 1]) ++rr;
+    const int s0 = bm.cseg[rr], s1 = bm.cseg[rr + 1];
+    if (s1 - s0 > kSmallSeg) continue;
+    const uint32_t key = keys[i];
+    int rank = 0;
+    for (int j = s0; j < s1; ++j) rank += keys[j] < key;
+    const int64_t o = bm.cbase[rr] + rank;
+    C_col[o] = (int32_t)key;
+    C_val[o] = vals[i];
+  }
+  for (int r = 0; r < nr; ++r) {
+    const int s0 = bm.cseg[r], s1 = bm.cseg[r + 1];
+    if (s1 - s0 <= kSmallSeg) continue;
+    __syncthreads();
+    smem_bitonic_sort<T, V>(keys + s0, vals + s0, s1 - s0);
+    const int64_t o = bm.cbase[r];
+    for (int i = tid; i < s1 - s0; i += T) {
+      C_col[o + i] = (int32_t)keys[s0 + i];
+      C_val[o + i] = vals[s0 + i];
+    }
+  }
+}
+
+template <int CFG, int PASS, typename V>
+__device__ __noinline__ void dense_row(const SpgemmArgs<V>& p, BlockMeta& bm, int b0, unsigned char* smem, int* chist);
 
 // -----------------------------------------------------------------------------------
 // The per-configuration kernel.  PASS 0 = symbolic, 1 = numeric.
@@ -605,48 +686,22 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
           // ordered map: write every entry at (occupied slots before its cluster) + (rank in
           // the cluster) — the row comes out sorted without moving anything in shared memory
           const int64_t ob = bm.cbase[r];
+          sort_runs<V>(rk, rv, S, (uint32_t)lane, 32u);
+          __syncwarp();
           int before = 0;
-          for (uint32_t c0 = 0; c0 < S; c0 += 32) ordered_chunk_emit<V>(rk, rv, S, c0, before, ob, p.C_col, p.C_val);
-        } else {
-          // a probing run wrapped around: compact the region in place, then sort and write
-          int pos = 0;
           for (uint32_t c0 = 0; c0 < S; c0 += 32) {
             const uint32_t s = c0 + lane;
-            uint32_t kk = kEmptyKey;
-            V vv = V(0);
-            if (s < S) { kk = rk[s]; vv = rv[s]; }
+            const uint32_t kk = s < S ? rk[s] : kEmptyKey;
             const uint32_t occ = __ballot_sync(0xffffffffu, kk != kEmptyKey);
-            __syncwarp();
             if (kk != kEmptyKey) {
-              const int o = pos + __popc(occ & ((1u << lane) - 1u));
-              rk[o] = kk;
-              rv[o] = vv;
+              const int64_t o = ob + before + __popc(occ & ((1u << lane) - 1u));
+              p.C_col[o] = (int32_t)kk;
+              p.C_val[o] = rv[s];
             }
-            pos += __popc(occ);
-            __syncwarp();
+            before += __popc(occ);
           }
-          const int cnt = pos;
-          const int64_t ob = bm.cbase[r];
-          if (cnt <= kSmallSeg) {
-            // rank counting: all lanes read key j together (smem broadcast)
-            for (int e0 = 0; e0 < cnt; e0 += 32) {
-              const int e = e0 + lane;
-              const uint32_t key = e < cnt ? rk[e] : 0xffffffffu;
-              const V val = e < cnt ? rv[e] : V(0);
-              int rank = 0;
-              for (int j = 0; j < cnt; ++j) rank += rk[j] < key;
-              if (e < cnt) {
-                p.C_col[ob + rank] = (int32_t)key;
-                p.C_val[ob + rank] = val;
-              }
-            }
-          } else {
-            smem_bitonic_sort<32, V, true>(rk, rv, cnt);
-            for (int e = lane; e < cnt; e += 32) {
-              p.C_col[ob + e] = (int32_t)rk[e];
-              p.C_val[ob + e] = rv[e];
-            }
-          }
+        } else {
+          warp_row_sorted_write<V>(rk, rv, S, bm.cbase[r], p.C_col, p.C_val);
         }
         __syncwarp();
       }
@@ -717,52 +772,27 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
                                     bm.scan_part);
         }
       } else {
-        // ---- compaction (order preserving -> row regions stay in row order) ----
-        int64_t running = 0;
-        for (uint32_t base = 0; base < capt; base += T) {
-          const uint32_t s = base + tid;
-          uint32_t kk = kEmptyKey;
-          V vv = V(0);
-          if (s < capt) { kk = keys[s]; vv = vals[s]; }
-          const int64_t fl = kk != kEmptyKey;
-          int64_t tot;
-          const int64_t pos = block_excl_scan<T>(fl, bm.scan_part, &tot);
-          if (fl) { keys[running + pos] = kk; vals[running + pos] = vv; }
-          running += tot;
-          __syncthreads();
-        }
-        // ---- short rows: rank counting, written straight to C ----
-        const int ncnt = (int)bm.cnt;
-        {
-          int rr = 0;
-          for (int i = tid; i < ncnt; i += T) {
-            while (i >= bm.cseg[rr + 1]) ++rr;
-            const int s0 = bm.cseg[rr], s1 = bm.cseg[rr + 1];
-            if (s1 - s0 > kSmallSeg) continue;
-            const uint32_t key = keys[i];
-            int rank = 0;
-            for (int j = s0; j < s1; ++j) rank += keys[j] < key;
-            const int64_t o = bm.cbase[rr] + rank;
-            p.C_col[o] = (int32_t)key;
-            p.C_val[o] = vals[i];
-          }
-        }
-        // ---- long rows: bitonic sort in shared memory, then coalesced write ----
-        for (int rr = 0; rr < nr; ++rr) {
-          const int s0 = bm.cseg[rr], s1 = bm.cseg[rr + 1];
-          if (s1 - s0 <= kSmallSeg) continue;
-          __syncthreads();
-          smem_bitonic_sort<T, V>(keys + s0, vals + s0, s1 - s0);
-          const int64_t o = bm.cbase[rr];
-          for (int i = tid; i < s1 - s0; i += T) {
-            p.C_col[o + i] = (int32_t)keys[s0 + i];
-            p.C_val[o + i] = vals[s0 + i];
-          }
-        }
+        block_sorted_write<T, V>(keys, vals, capt, bm, p.C_col, p.C_val);
       }
     } else {
-      // ============================ DENSE ACCUMULATOR =============================
-      // single row; windows over [colmin, colmax] (Fig. 5)
+      dense_row<CFG, PASS, V>(p, bm, b0, smem, chist);
+    }
+    __syncthreads();
+    b0 = b1;
+  }
+}
+
+// ============================ DENSE ACCUMULATOR (single row) =============================
+// Windows over [colmin, colmax] (Fig. 5); kept out of line so the hash paths'
+// hot loops stay compact in the instruction cache.
+template <int CFG, int PASS, typename V>
+__device__ __noinline__ void dense_row(const SpgemmArgs<V>& p, BlockMeta& bm, int b0, unsigned char* smem, int* chist) {
+  constexpr int T = kCfgThreads[CFG];
+  constexpr int NW = T / 32;
+  const int tid = threadIdx.x;
+  const int64_t nnzA = bm.nnzA;
+  {
+    {
       const int32_t row = bm.row[b0];
       // symbolic windows start 32-aligned so a bitmap word never straddles a 2^15 chunk
       const int64_t lo = PASS == 0 ? (bm.colmin & ~31) : bm.colmin, hi = bm.colmax;
@@ -827,8 +857,6 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
         for (int i = tid; i < p.nchunks; i += T) dst[i] = chist[i];
       }
     }
-    __syncthreads();
-    b0 = b1;
   }
 }
 
