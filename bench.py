@@ -34,6 +34,8 @@ sys.path.insert(0, ROOT)
 
 import workloads as W  # noqa: E402
 
+dist = sdist = None      # torch.distributed / the row partitioner, bound at N>1
+
 WORKLOAD_NAMES = {
     "c1": "C1 2-D 5-point Poisson 64x64, A*A, fp64",
     "c2": "C2 3-D 27-point 128^3 AMG Galerkin R*(A*P): two SpGEMMs, fp64",
@@ -172,12 +174,19 @@ def run_speck(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.dist_backend == "gloo":
+        # host-staged collectives; lets the N>1 logic run with several ranks on one GPU (testing)
+        local_rank %= torch.cuda.device_count()
     torch.cuda.set_device(local_rank)
     dev = torch.device("cuda", local_rank)
     if world > 1:
+        global dist, sdist
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=dev)
         from paper_conf_ppopp_pargerwms20_b200 import dist as sdist
+        if args.dist_backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group("gloo")
 
     cfg = args.config
     t_gen = time.time()
@@ -192,30 +201,27 @@ def run_speck(args):
 
     state = {}
 
-    def one_step():
+    def compute(pairs, hs):
+        """One pass of the hot path over `pairs` [(A, B)]; B=None means the previous result."""
         if world == 1:
             if cfg == "c2":
-                (_, A, P), (_, R, _) = probs
-                AP = handles[0].spgemm(A, P)
-                Ac = handles[1].spgemm(R, AP)
-                state["out"] = (AP, Ac)
-                return Ac
-            (_, A, B), = probs
-            C = handles[0].spgemm(A, B)
-            state["out"] = (C,)
-            return C
+                (A, P), (R, _) = pairs
+                AP = hs[0].spgemm(A, P)
+                return (AP, hs[1].spgemm(R, AP))
+            (A, B), = pairs
+            return (hs[0].spgemm(A, B),)
         # multi-GPU: row-sharded, B replicated
         if cfg == "c2":
-            (_, A, P), (_, R, _) = probs
-            blk = sdist.spgemm_rowsharded(A, P, local=handles[0].spgemm, bounds=state["bounds"][0])
+            (A, P), (R, _) = pairs
+            blk = sdist.spgemm_rowsharded(A, P, local=hs[0].spgemm, bounds=state["bounds"][0])
             AP = sdist.allgather_csr(blk, A.rows)
-            blk2 = sdist.spgemm_rowsharded(R, AP, local=handles[1].spgemm, bounds=state["bounds"][1])
-            state["out"] = (blk, blk2)
-            return blk2
-        (_, A, B), = probs
-        blk = sdist.spgemm_rowsharded(A, B, local=handles[0].spgemm, bounds=state["bounds"][0])
-        state["out"] = (blk,)
-        return blk
+            return (blk, sdist.spgemm_rowsharded(R, AP, local=hs[1].spgemm, bounds=state["bounds"][1]))
+        (A, B), = pairs
+        return (sdist.spgemm_rowsharded(A, B, local=hs[0].spgemm, bounds=state["bounds"][0]),)
+
+    def one_step():
+        state["out"] = compute([(A, B) for (_, A, B) in probs], handles)
+        return state["out"][-1]
 
     if world > 1:
         # balanced product split (Alg. 1 on the replicated A; identical on every rank) — untimed
@@ -319,8 +325,8 @@ def run_speck(args):
 
     # ---- end-to-end through the public API with host buffers (rank 0, N=1)
     e2e = None
-    if world == 1 and not args.no_e2e:
-        e2e = run_e2e(sp, cfg, probs, dev, min(args.steps, 5), step_products)
+    if not args.no_e2e:
+        e2e = run_e2e(sp, probs, dev, min(args.steps, 5), step_products, compute, world)
 
     # ---- CPU baseline: the oracle on this host's cores (rank 0, N=1)
     cpu = None
@@ -359,8 +365,10 @@ def run_speck(args):
         dist.destroy_process_group()
 
 
-def run_e2e(sp, cfg, probs, dev, steps, step_products):
-    """Same metric through the public API, host (pinned) inputs in, host result out."""
+def run_e2e(sp, probs, dev, steps, step_products, compute, world):
+    """Same metric through the public API, host (pinned) inputs in, host result out.  At N>1
+    every rank copies the replicated inputs and reads back its own row block of the result;
+    the time is the max over ranks."""
     host_in = []
     for (label, A, B) in probs:
         host_in.append(tuple(None if M is None else W.CSR(M.rows, M.cols, M.row_ptr.cpu().pin_memory(),
@@ -376,6 +384,8 @@ def run_e2e(sp, cfg, probs, dev, steps, step_products):
     times, bo = [], 0
     for it in range(steps + 1):
         torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         a.record(stream)
         for pair_h, pair_d in zip(host_in, dev_in):
@@ -385,13 +395,7 @@ def run_e2e(sp, cfg, probs, dev, steps, step_products):
                 Md.row_ptr.copy_(Mh.row_ptr, non_blocking=True)
                 Md.col.copy_(Mh.col, non_blocking=True)
                 Md.val.copy_(Mh.val, non_blocking=True)
-        if cfg == "c2":
-            (A, P), (R, _) = dev_in
-            AP = h[0].spgemm(A, P)
-            C = h[1].spgemm(R, AP)
-        else:
-            (A, B), = dev_in
-            C = h[0].spgemm(A, B)
+        C = compute(dev_in, h)[-1]
         res = [torch.empty(t.shape, dtype=t.dtype, pin_memory=True) for t in (C.row_ptr, C.col, C.val)]
         for r, t in zip(res, (C.row_ptr, C.col, C.val)):
             r.copy_(t, non_blocking=True)
@@ -401,6 +405,10 @@ def run_e2e(sp, cfg, probs, dev, steps, step_products):
         if it > 0:                                     # first iteration warms the handles
             times.append(a.elapsed_time(b))
     ms = statistics.mean(times)
+    if world > 1:
+        t = torch.tensor([ms], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
     return {"value": round(2.0 * step_products / (ms * 1e-3) / 1e9, 3), "unit": "GFLOP/s",
             "h2d_bytes_per_step": int(bi), "d2h_bytes_per_step": int(bo), "ms_per_step": round(ms, 3)}
 
@@ -443,6 +451,8 @@ def main():
     ap.add_argument("--config", default="c2", choices=sorted(WORKLOAD_NAMES))
     ap.add_argument("--impl", default="speck", choices=["speck", "reference"])
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
+                    help="process-group backend for N>1 (gloo: testing several ranks on one GPU)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--opt", action="append", default=[], help="library option name=value (experiments)")
     ap.add_argument("--cpu-budget", type=float, default=20.0, help="seconds of oracle work for the CPU baseline")

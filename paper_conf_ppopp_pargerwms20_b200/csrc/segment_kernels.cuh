@@ -2,12 +2,13 @@
 //
 // The paper processes a row that needs the largest kernel with windowed dense accumulation,
 // one window after the other inside one block.  B200 keeps that
-// for rows whose window overhead is small ("windows" jobs: one CTA, dense windows of 55.6K
-// (fp32) / 27.7K (fp64) columns, resume positions per referenced B row), and splits the
-// others into *column segments*: consecutive 2^s-column chunks grouped so that each
-// segment's exact size (from the per-chunk counts the symbolic pass recorded) fits the
-// largest hash map at <= 66% fill (ordered hash, sorted write-out), or a single chunk that is
-// accumulated densely.  Segments of one row are independent CTAs writing disjoint, known
+// for rows whose window overhead is small ("windows" jobs: one CTA of configuration kSegCfg,
+// dense windows of that configuration's shared memory, each referenced B row located in the
+// window by binary search), and splits the others into *column segments*: consecutive
+// 2^s-column chunks grouped so that each segment's exact size (from the per-chunk counts the
+// symbolic pass recorded) fits the kSegCfg hash map at the ordered fill (ordered hash, sorted
+// write-out), or a single chunk that is accumulated densely.  kSegCfg = 3 (512 threads,
+// 2 CTAs/SM) so two jobs share an SM and one job's barriers hide behind the other's work.  Segments of one row are independent CTAs writing disjoint, known
 // ranges of the row, so a long, wide, sparse row (C5) or one of a few giant rows (C4) is
 // spread over many SMs.
 #pragma once
@@ -155,7 +156,7 @@ __device__ int64_t dense_window_pass(const SpgemmArgs<V>& p, int64_t a0, int ale
   return dense_emit<T, V>(bits, dvals, nwords, wlo, out, p.C_col, p.C_val, part);
 }
 
-// One CTA (the largest configuration, 1 CTA/SM) per job.
+// One CTA of configuration kSegCfg (2 CTAs/SM) per job.
 template <typename V>
 __global__ void __launch_bounds__(kCfgThreads[kSegCfg], 1024 / kCfgThreads[kSegCfg])
     k_segments(SpgemmArgs<V> p, const Seg* __restrict__ segs) {
