@@ -15,6 +15,8 @@ namespace speck {
 // reduction produces prods_r, prods_r,max, colmin, colmax.  Global Σprods / max prods and
 // the #single-NZ / #empty rows go to the stats block with one atomic per CTA.
 // ------------------------------------------------------------------------------------
+constexpr int kAnaU = 4;   // NZ per lane per iteration of the analysis
+
 template <int GA>
 __global__ void __launch_bounds__(256) k_analysis(const int64_t* __restrict__ A_rp, const int32_t* __restrict__ A_col,
                                                   const int64_t* __restrict__ B_rp, const int32_t* __restrict__ B_col,
@@ -40,15 +42,27 @@ __global__ void __launch_bounds__(256) k_analysis(const int64_t* __restrict__ A_
     }
     int64_t p = 0;
     int32_t ml = 0, cmin = INT_MAX, cmax = -1;
-    for (int64_t q = a0 + sub; q < a1; q += GA) {
-      const int32_t k = A_col[q];
-      const int64_t b0 = B_rp[k], b1 = B_rp[k + 1];
-      const int64_t len = b1 - b0;
-      p += len;
-      ml = max(ml, (int32_t)len);
-      if (len > 0) {
-        cmin = min(cmin, B_col[b0]);
-        cmax = max(cmax, B_col[b1 - 1]);
+    // kAnaU NZ per lane per iteration, each stage's loads issued together (the A col ->
+    // B row_ptr -> B col chain is three dependent round trips; unrolling overlaps them)
+    for (int64_t q = a0 + sub; q < a1; q += GA * kAnaU) {
+      int32_t k[kAnaU];
+      int64_t b0[kAnaU], b1[kAnaU];
+#pragma unroll
+      for (int u = 0; u < kAnaU; ++u) k[u] = q + u * GA < a1 ? A_col[q + u * GA] : -1;
+#pragma unroll
+      for (int u = 0; u < kAnaU; ++u) {
+        b0[u] = k[u] >= 0 ? B_rp[k[u]] : 0;
+        b1[u] = k[u] >= 0 ? B_rp[k[u] + 1] : 0;
+      }
+#pragma unroll
+      for (int u = 0; u < kAnaU; ++u) {
+        const int64_t len = b1[u] - b0[u];
+        p += len;
+        ml = max(ml, (int32_t)len);
+        if (len > 0) {
+          cmin = min(cmin, B_col[b0[u]]);
+          cmax = max(cmax, B_col[b1[u] - 1]);
+        }
       }
     }
 #pragma unroll

@@ -138,7 +138,7 @@ int pow2_clamp(double x, int lo, int hi) {
   return p;
 }
 
-// Row analysis (Alg. 1): GA lanes per row (GA ~ average row length of A), rows longer than
+// Row analysis (Alg. 1): GA lanes per row (GA x kAnaU ~ average row length of A), rows longer than
 // kAnaLong deferred to one CTA each.  `st` may be null (no statistics).
 speck_status_t run_analysis(speck_handle_t h, const speck_csr_t* A, const speck_csr_t* B, int64_t* prods,
                             int32_t* maxlen, int32_t* colmin, int32_t* colmax, AnalysisStats* st, cudaStream_t s) {
@@ -149,7 +149,7 @@ speck_status_t run_analysis(speck_handle_t h, const speck_csr_t* A, const speck_
   unsigned* nlong = reinterpret_cast<unsigned*>(static_cast<char*>(h->small.p) + 640);
   int32_t* lrows = static_cast<int32_t*>(h->ana_long.p);
   CK(cudaMemsetAsync(nlong, 0, 4, s));
-  const int ga = pow2_clamp(m > 0 ? (double)A->nnz / (double)m : 1.0, 1, 32);
+  const int ga = pow2_clamp(m > 0 ? (double)A->nnz / (double)m / kAnaU : 1.0, 1, 32);   // GA*kAnaU ~ avg row
   const unsigned agrid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((m * ga + 255) / 256, (int64_t)h->num_sms * 8));
 #define SPECK_ANA(GA)                                                                                        \
   k_analysis<GA><<<agrid, 256, 0, s>>>(A->row_ptr, A->col_idx, B->row_ptr, B->col_idx, m, prods, maxlen, colmin, \

@@ -103,30 +103,53 @@ __device__ __forceinline__ uint32_t probe_insert_mono(uint32_t* keys, uint32_t S
   }
 }
 
-// Sort every probing run of an ordered map region in place (keys and values): the thread
-// owning a run's first slot walks the run and insertion-sorts it (runs are short and nearly
-// sorted).  Threads t0, t0+step, ... examine the slots.  After this (and a barrier), the
-// occupied slots are in column order, so the write-out is a plain order-preserving compaction.
+// Sorted write-out of the slots [w0, w1) of an ordered map region rk/rv[0, S) by one warp,
+// without moving anything in shared memory.  With monotone homes and no wrap-around, every
+// occupied slot s lies in a probing run [rs, re) (maximal occupied range) that holds exactly
+// the keys homed inside it, and runs appear in column order; so the sorted position of slot s
+// is (#occupied before rs) + #{j in [rs, re) : key_j < key_s}, where
+// #occupied before rs = #occupied before s - (s - rs).  Run bounds come from the window's
+// occupancy ballot (a short walk only for runs crossing a window edge); the rank loop is as
+// long as the window's longest run.  `before` = #occupied slots of the region before w0.
+// Returns the number of entries written.
 template <typename V>
-__device__ __forceinline__ void sort_runs(uint32_t* keys, V* vals, uint32_t S, uint32_t t0, uint32_t step) {
-  for (uint32_t s = t0; s < S; s += step) {
-    if (keys[s] == kEmptyKey || (s > 0 && keys[s - 1] != kEmptyKey)) continue;   // not a run start
-    uint32_t e = s + 1;
-    while (e < S && keys[e] != kEmptyKey) ++e;
-    for (uint32_t i = s + 1; i < e; ++i) {
-      const uint32_t k = keys[i];
-      if (keys[i - 1] <= k) continue;
-      const V v = vals[i];
-      uint32_t j = i;
-      while (j > s && keys[j - 1] > k) {
-        keys[j] = keys[j - 1];
-        vals[j] = vals[j - 1];
-        --j;
+__device__ __forceinline__ int warp_write_ordered(const uint32_t* rk, const V* rv, uint32_t S, uint32_t w0, uint32_t w1,
+                                                  int64_t ob, int before, int32_t* __restrict__ C_col,
+                                                  V* __restrict__ C_val) {
+  const int lane = lane_id();
+  const uint32_t lt = (1u << lane) - 1u;
+  const uint32_t gt = ~(lt | (1u << lane));
+  // occupied slots immediately before the window (a run entering it from the left)
+  uint32_t carry = 0;
+  if (w0 > 0 && w0 < w1 && rk[w0] != kEmptyKey)
+    while (carry < w0 && rk[w0 - 1 - carry] != kEmptyKey) ++carry;
+  int written = 0;
+  for (uint32_t c0 = w0; c0 < w1; c0 += 32) {
+    const uint32_t s = c0 + lane;
+    const uint32_t k = s < S ? rk[s] : kEmptyKey;        // slots past w1 only bound runs
+    const uint32_t occ = __ballot_sync(0xffffffffu, k != kEmptyKey);
+    const uint32_t mine = occ & (w1 - c0 >= 32 ? 0xffffffffu : ((1u << (w1 - c0)) - 1u));
+    if ((mine >> lane) & 1u) {
+      const uint32_t zb = ~occ & lt;
+      const uint32_t rs = zb ? c0 + 32 - __clz(zb) : c0 - carry;
+      const uint32_t za = ~occ & gt;
+      uint32_t re;
+      if (za) {
+        re = c0 + __ffs(za) - 1;
+      } else {
+        re = c0 + 32;
+        while (re < S && rk[re] != kEmptyKey) ++re;
       }
-      keys[j] = k;
-      vals[j] = v;
+      int rank = 0;
+      for (uint32_t j = rs; j < re; ++j) rank += rk[j] < k;
+      const int64_t o = ob + before + written + __popc(occ & lt) - (int)(s - rs) + rank;
+      C_col[o] = (int32_t)k;
+      C_val[o] = rv[s];
     }
+    written += __popc(mine);
+    carry = occ == 0xffffffffu ? carry + 32 : __clz(~occ);
   }
+  return written;
 }
 
 // symbolic insert: true if the key was new
@@ -178,18 +201,16 @@ __device__ __noinline__ void smem_bitonic_sort(uint32_t* keys, V* vals, int n) {
   }
 }
 
-// Block-wide write-out of one ordered map region [0, S): sort the probing runs in place,
-// then an order-preserving compaction — warp-contiguous slot ranges, one block-level prefix
-// of the per-warp occupancy, coalesced writes.  Barriers inside; `part` = >= 32 int64 scratch.
+// Block-wide write-out of one ordered map region [0, S): warp-contiguous slot ranges, one
+// block-level prefix of the per-warp occupancy, then warp_write_ordered per range (runs may
+// cross range edges; slots are only read).  Barriers inside; `part` = >= 32 int64 scratch.
 template <int T, typename V>
-__device__ void block_write_ordered(uint32_t* rk, V* rv, uint32_t S, int64_t ob, int32_t* __restrict__ C_col,
+__device__ void block_write_ordered(const uint32_t* rk, const V* rv, uint32_t S, int64_t ob, int32_t* __restrict__ C_col,
                                     V* __restrict__ C_val, int64_t* part) {
   constexpr int NW = T / 32;
   const int lane = lane_id(), wp = warp_id();
-  sort_runs<V>(rk, rv, S, threadIdx.x, T);
   const uint32_t SW = ((S + NW - 1) / NW + 31u) & ~31u;
   const uint32_t w0 = min(S, wp * SW), w1 = min(S, w0 + SW);
-  __syncthreads();
   int cw = 0;
   for (uint32_t c0 = w0; c0 < w1; c0 += 32) {
     const uint32_t s = c0 + lane;
@@ -199,17 +220,7 @@ __device__ void block_write_ordered(uint32_t* rk, V* rv, uint32_t S, int64_t ob,
   __syncthreads();
   int before = 0;
   for (int w = 0; w < wp; ++w) before += (int)part[w];
-  for (uint32_t c0 = w0; c0 < w1; c0 += 32) {
-    const uint32_t s = c0 + lane;
-    const uint32_t kk = s < w1 ? rk[s] : kEmptyKey;
-    const uint32_t occ = __ballot_sync(0xffffffffu, kk != kEmptyKey);
-    if (kk != kEmptyKey) {
-      const int64_t o = ob + before + __popc(occ & ((1u << lane) - 1u));
-      C_col[o] = (int32_t)kk;
-      C_val[o] = rv[s];
-    }
-    before += __popc(occ);
-  }
+  warp_write_ordered<V>(rk, rv, S, w0, w1, ob, before, C_col, C_val);
   __syncthreads();
 }
 
@@ -685,21 +696,7 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
         } else if (ordered && !__any_sync(0xffffffffu, wrapped)) {
           // ordered map: write every entry at (occupied slots before its cluster) + (rank in
           // the cluster) — the row comes out sorted without moving anything in shared memory
-          const int64_t ob = bm.cbase[r];
-          sort_runs<V>(rk, rv, S, (uint32_t)lane, 32u);
-          __syncwarp();
-          int before = 0;
-          for (uint32_t c0 = 0; c0 < S; c0 += 32) {
-            const uint32_t s = c0 + lane;
-            const uint32_t kk = s < S ? rk[s] : kEmptyKey;
-            const uint32_t occ = __ballot_sync(0xffffffffu, kk != kEmptyKey);
-            if (kk != kEmptyKey) {
-              const int64_t o = ob + before + __popc(occ & ((1u << lane) - 1u));
-              p.C_col[o] = (int32_t)kk;
-              p.C_val[o] = rv[s];
-            }
-            before += __popc(occ);
-          }
+          warp_write_ordered<V>(rk, rv, S, 0u, S, bm.cbase[r], 0, p.C_col, p.C_val);
         } else {
           warp_row_sorted_write<V>(rk, rv, S, bm.cbase[r], p.C_col, p.C_val);
         }

@@ -31,6 +31,10 @@ def main(rep, launch=0):
         if k in h:
             i = h.index(k)
             print(f"  {k:70s} {d[i]:>20s} {units[i]}")
+    stalls = [(float(d[i] or 0), k) for i, k in enumerate(h)
+              if k.startswith("smsp__pcsamp_warps_issue_stalled_") and not k.endswith("_not_issued")]
+    tot = sum(v for v, _ in stalls) or 1.0
+    print("stall reasons (pc sampling):", ", ".join(f"{k[33:]} {100 * v / tot:.1f}%" for v, k in sorted(stalls, reverse=True)[:8]))
     src = list(csv.reader(io.StringIO(ncu([rep, "--page", "source", "--csv", "--print-source", "cuda,sass",
                                            "--launch-skip", str(launch), "--launch-count", "1"]))))
     cur, hdr, out = None, None, []
