@@ -61,6 +61,7 @@ struct speck_handle_s {
   int64_t launches = 0;  // kernels launched by this handle (cumulative)
   // long-row segments
   int64_t opt_segments = 1;
+  int64_t opt_warp_rows = 1;
   bool seg_enabled = false;
   int seg_shift = 15, nchunks = 0;
   int64_t long_thr = INT64_MAX, n_cand = 0, n_segs = 0, cand_start = 0;
@@ -204,6 +205,8 @@ speck_status_t set_smem_attrs(speck_handle_t h) {
     for (int pass = 0; pass < 2; ++pass)
       CK(cudaFuncSetAttribute(spgemm_fn<V>(c, pass), cudaFuncAttributeMaxDynamicSharedMemorySize, kCfgMapBytes[c]));
   CK(cudaFuncSetAttribute(k_segments<V>, cudaFuncAttributeMaxDynamicSharedMemorySize, kCfgMapBytes[kSegCfg]));
+  CK(cudaFuncSetAttribute(k_warp_rows<0, V>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytes * (kWarpRowThreads / 32)));
+  CK(cudaFuncSetAttribute(k_warp_rows<1, V>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytes * (kWarpRowThreads / 32)));
   return SPECK_OK;
 }
 
@@ -234,6 +237,25 @@ speck_status_t join(speck_handle_t h, cudaStream_t s, int n) {
   return SPECK_OK;
 }
 
+int64_t warp_row_fill(speck_handle_t h, int pass) {
+  if (pass == 0) return wr_sym_fill();
+  return h->dtype == SPECK_F64 ? wr_num_fill<double>() : wr_num_fill<float>();
+}
+
+// Small-row kernel: persistent CTAs of 8 warps pulling rows from a counter (zeroed here).
+template <typename V>
+speck_status_t launch_warp_rows(speck_handle_t h, int pass, const SpgemmArgs<V>& a, cudaStream_t s) {
+  if (a.n_entries <= 0) return SPECK_OK;
+  unsigned long long* ctr = reinterpret_cast<unsigned long long*>(static_cast<char*>(h->small.p) + 1024 + 8 * pass);
+  CK(cudaMemsetAsync(ctr, 0, 8, s));
+  const int64_t grid = std::min<int64_t>((a.n_entries + 7) / 8, (int64_t)h->num_sms * kWarpRowCtasPerSM);
+  const size_t smem = (size_t)kWarpRegionBytes * (kWarpRowThreads / 32);
+  if (pass == 0) k_warp_rows<0, V><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
+  else k_warp_rows<1, V><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
+  CKL();
+  return SPECK_OK;
+}
+
 BinParams make_bin_params(speck_handle_t h, int pass) {
   BinParams bp{};
   bp.pass = pass;
@@ -243,6 +265,8 @@ BinParams make_bin_params(speck_handle_t h, int pass) {
     if (pass == 0) bp.cap[c] = sym_map_fill(c);
     else bp.cap[c] = h->dtype == SPECK_F64 ? num_map_fill<double>(c) : num_map_fill<float>(c);
   }
+  // smallest bin = rows of one warp (k_warp_rows) instead of merged blocks of configuration 0
+  if (h->opt_warp_rows) bp.cap[0] = warp_row_fill(h, pass);
   if (h->seg_enabled) {
     // every row that may exceed the largest numeric map is a symbolic cfg4 row, so that the
     // symbolic pass records its per-chunk counts; such rows become numeric segments
@@ -340,6 +364,9 @@ speck_status_t run_pass(speck_handle_t h, int pass, int lb, const int64_t* cat_s
     BinParams own = bp;
     for (int c = 0; c < kNumCfg; ++c)
       own.cap[c] = pass == 0 ? (int64_t)sym_map_fill(c) : (int64_t)num_map_fill<V>(c);
+    a.rows = nullptr;
+    a.n_entries = m;
+    if (h->opt_warp_rows && need_max <= warp_row_fill(h, pass)) return launch_warp_rows<V>(h, pass, a, s);
     int cfg = -1, R = 1;
     for (int c = 0; c < kNumCfg; ++c)
       if (need_max * kMaxGroupRows <= own.cap[c]) { cfg = c; R = kMaxGroupRows; break; }
@@ -383,6 +410,12 @@ speck_status_t run_pass(speck_handle_t h, int pass, int lb, const int64_t* cat_s
     SpgemmArgs<V> b = a;
     b.rows = bins + cat_start[cat];
     b.n_entries = n;
+    if (c == 0 && h->opt_warp_rows) {
+      st = launch_warp_rows<V>(h, pass, b, h->streams[si]);
+      if (st) return st;
+      si = (si + 1) % ns;
+      continue;
+    }
     if (c == 0) {
       b.group_rows = kMaxGroupRows;
       b.merge = 1;
@@ -787,6 +820,7 @@ speck_status_t speck_set_option(speck_handle_t h, int option, int64_t v) {
       if (v < 1 || v > kMaxStreams) return fail(h, SPECK_ERR_INVALID_ARGUMENT, "CONCURRENT_STREAMS must be 1..8");
       h->opt_streams = v; break;
     case SPECK_OPT_SEGMENTS: h->opt_segments = v; break;
+    case SPECK_OPT_WARP_ROWS: h->opt_warp_rows = v; break;
     default: return fail(h, SPECK_ERR_INVALID_ARGUMENT, "unknown option %d", option);
   }
   return SPECK_OK;

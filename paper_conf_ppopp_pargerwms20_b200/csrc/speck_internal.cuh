@@ -100,6 +100,23 @@ __host__ __device__ inline int64_t num_dense_window(int cfg) {
   return ((int64_t)(cfg_map_bytes(cfg) - 16) * 8 / (8 * (int64_t)sizeof(V) + 1)) & ~int64_t(31);
 }
 
+// Small rows: one warp per row in a private region (k_warp_rows).  8 warps x 7 KB per CTA and
+// 4 CTAs per SM = 1024 resident threads and the whole 228 KB; a row belongs here when its need
+// fits the region at the pass's fill.
+constexpr int kWarpRowThreads = 256;
+constexpr int kWarpRegionBytes = 7168;
+constexpr int kWarpRowCtasPerSM = 4;
+constexpr int kWarpRowChunk = 8;     // rows a warp claims per counter increment
+static_assert((kWarpRegionBytes * (kWarpRowThreads / 32) + 1024) * kWarpRowCtasPerSM <= kSmemPerSM, "warp-row CTAs");
+__host__ __device__ inline uint32_t wr_sym_cap() { return (uint32_t)(kWarpRegionBytes / 4); }
+__host__ __device__ inline uint32_t wr_sym_fill() { return (uint32_t)((uint64_t)wr_sym_cap() * kFillNum / 100); }
+template <typename V>
+__host__ __device__ inline uint32_t wr_num_cap() { return (uint32_t)((kWarpRegionBytes - 16) / num_slot_bytes<V>()); }
+template <typename V>
+__host__ __device__ inline uint32_t wr_num_val_offset() { return (wr_num_cap<V>() * 4u + 15u) & ~15u; }
+template <typename V>
+__host__ __device__ inline uint32_t wr_num_fill() { return (uint32_t)((uint64_t)wr_num_cap<V>() * kFillOrdered / 100); }
+
 // ----------------------------------------------------------------------------------
 // Analysis statistics block written by the analysis kernel (read back once, sync #1).
 // ----------------------------------------------------------------------------------

@@ -522,6 +522,54 @@ __device__ __noinline__ void block_sorted_write(uint32_t* keys, V* vals, uint32_
   }
 }
 
+// One row of C by one warp in a private map region rk/rv[0, S) (cleared here): expand-balanced
+// products, hash insert (symbolic: count new keys; numeric: equal keys of a warp step add in
+// rounds — the region is private, so no atomics on values), then the sorted write-out
+// (ordered map for rows > kSmallSeg entries, else rank counting).  Returns the symbolic count.
+template <int PASS, typename V>
+__device__ __forceinline__ int warp_row(const SpgemmArgs<V>& p, uint32_t* rk, V* rv, uint32_t S, int64_t a0, int alen,
+                                        int32_t cmin, int32_t cmax, int32_t cnt, int64_t cbase) {
+  const int lane = lane_id();
+  for (uint32_t i = lane; i < S; i += 32) {
+    rk[i] = kEmptyKey;
+    if (PASS == 1) rv[i] = V(0);
+  }
+  __syncwarp();
+  const uint32_t mlo = (uint32_t)cmin;
+  const uint64_t mmult = mono_mult((uint32_t)(cmax - cmin + 1), S);
+  // long rows use the order-preserving map (sorted write-out without a sort network);
+  // short rows keep the scrambled hash (robust to clustered columns) and rank counting
+  const bool ordered = PASS == 1 && cnt > kSmallSeg;
+  int newc = 0, wrapped = 0;
+  expand_row<PASS, V>(p, a0, alen, 0, 1, [&](uint32_t col, V v, bool act) {
+    if (PASS == 0) {
+      if (act) newc += hash_insert_key(rk, S, col);
+    } else {
+      const uint32_t peers = __match_any_sync(0xffffffffu, col);
+      const uint32_t lt = (1u << lane_id()) - 1u;
+      uint32_t s = 0;
+      if (act && !(peers & lt))
+        s = probe_insert_mono(rk, S, ordered ? mono_slot(col, mlo, mmult) : hash_slot(col, S), col, &wrapped);
+      s = __shfl_sync(0xffffffffu, s, __ffs(peers) - 1);   // the key's slot, from its first lane
+      const int rank = __popc(peers & lt);
+      const int maxg = (int)__reduce_max_sync(0xffffffffu, (unsigned)__popc(peers));
+      for (int t = 0; t < maxg; ++t) {
+        if (act && rank == t) rv[s] += v;
+        __syncwarp();
+      }
+    }
+  });
+  if (PASS == 0) return warp_sum(newc);
+  if (ordered && !__any_sync(0xffffffffu, wrapped)) {
+    // ordered map: every entry goes to (occupied slots before its run) + (rank in the run)
+    warp_write_ordered<V>(rk, rv, S, 0u, S, cbase, 0, p.C_col, p.C_val);
+  } else {
+    warp_row_sorted_write<V>(rk, rv, S, cbase, p.C_col, p.C_val);
+  }
+  __syncwarp();
+  return 0;
+}
+
 template <int CFG, int PASS, typename V>
 __device__ __noinline__ void dense_row(const SpgemmArgs<V>& p, BlockMeta& bm, int b0, unsigned char* smem, int* chist);
 
@@ -656,50 +704,9 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
       const int lane = lane_id();
       for (int r = warp_id(); r < nr; r += NW) {
         const uint32_t rb = bm.rbase[r], S = bm.rbase[r + 1] - rb;
-        uint32_t* rk = keys + rb;
-        V* rv = vals + rb;
-        for (uint32_t i = lane; i < S; i += 32) {
-          rk[i] = kEmptyKey;
-          if (PASS == 1) rv[i] = V(0);
-        }
-        __syncwarp();
-        const int64_t a0 = bm.astart[r];
-        const int alen = (int)(bm.aoff[r + 1] - bm.aoff[r]);
-        const uint32_t mlo = (uint32_t)bm.rlo[r];
-        const uint64_t mmult = mono_mult((uint32_t)(bm.rhi[r] - bm.rlo[r] + 1), S);
-        // long rows use the order-preserving map (sorted write-out without a sort network);
-        // short rows keep the scrambled hash (robust to clustered columns) and rank counting
-        const bool ordered = PASS == 1 && bm.cseg[r + 1] - bm.cseg[r] > kSmallSeg;
-        int newc = 0, wrapped = 0;
-        expand_row<PASS, V>(p, a0, alen, 0, 1, [&](uint32_t col, V v, bool act) {
-          if (PASS == 0) {
-            if (act) newc += hash_insert_key(rk, S, col);
-          } else {
-            const uint32_t peers = __match_any_sync(0xffffffffu, col);
-            const uint32_t lt = (1u << lane_id()) - 1u;
-            uint32_t s = 0;
-            if (act && !(peers & lt))
-              s = probe_insert_mono(rk, S, ordered ? mono_slot(col, mlo, mmult) : hash_slot(col, S), col, &wrapped);
-            s = __shfl_sync(0xffffffffu, s, __ffs(peers) - 1);   // the key's slot, from its first lane
-            // the region is private to this warp: equal keys add in rounds, no atomics
-            const int rank = __popc(peers & lt);
-            const int maxg = (int)__reduce_max_sync(0xffffffffu, (unsigned)__popc(peers));
-            for (int t = 0; t < maxg; ++t) {
-              if (act && rank == t) rv[s] += v;
-              __syncwarp();
-            }
-          }
-        });
-        if (PASS == 0) {
-          newc = warp_sum(newc);
-          if (lane == 0) p.cnt[bm.row[b0 + r]] = newc;
-        } else if (ordered && !__any_sync(0xffffffffu, wrapped)) {
-          // ordered map: write every entry at (occupied slots before its cluster) + (rank in
-          // the cluster) — the row comes out sorted without moving anything in shared memory
-          warp_write_ordered<V>(rk, rv, S, 0u, S, bm.cbase[r], 0, p.C_col, p.C_val);
-        } else {
-          warp_row_sorted_write<V>(rk, rv, S, bm.cbase[r], p.C_col, p.C_val);
-        }
+        const int c = warp_row<PASS, V>(p, keys + rb, vals + rb, S, bm.astart[r], (int)(bm.aoff[r + 1] - bm.aoff[r]),
+                                        bm.rlo[r], bm.rhi[r], bm.cseg[r + 1] - bm.cseg[r], bm.cbase[r]);
+        if (PASS == 0 && lane == 0) p.cnt[bm.row[b0 + r]] = c;
         __syncwarp();
       }
     } else if (!bm.dense) {
@@ -854,6 +861,80 @@ __device__ __noinline__ void dense_row(const SpgemmArgs<V>& p, BlockMeta& bm, in
         for (int i = tid; i < p.nchunks; i += T) dst[i] = chist[i];
       }
     }
+  }
+}
+
+// -----------------------------------------------------------------------------------
+// Small rows, one warp each (B200 replacement of the paper's block merge of small rows,
+// P:785-804): every warp owns a 7 KB region and pulls rows of the bin from a global counter
+// one row ahead, so no warp ever waits at a block barrier for another warp's row (ncu: 33% of
+// the stall samples of the merged-block kernel were barrier waits).  The region is sized to
+// the row (symbolic: products at 66% fill; numeric: exact nnz at 50%), so clearing and the
+// write-out scan only the slots a row can use.  Rows of the bin (p.rows) or, without global
+// load balancing, every row of A (p.rows == nullptr).
+// -----------------------------------------------------------------------------------
+template <int PASS, typename V>
+__global__ void __launch_bounds__(kWarpRowThreads, kWarpRowCtasPerSM)
+    k_warp_rows(SpgemmArgs<V> p, unsigned long long* __restrict__ counter) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  const int lane = lane_id();
+  unsigned char* region = smem + warp_id() * kWarpRegionBytes;
+  uint32_t* rk = reinterpret_cast<uint32_t*>(region);
+  V* rv = reinterpret_cast<V*>(region + (PASS == 0 ? 0u : wr_num_val_offset<V>()));
+  const uint32_t cap = PASS == 0 ? wr_sym_cap() : wr_num_cap<V>();
+  const int64_t n = p.n_entries;
+  // row metadata, one field per lane: 0 A_rp[r], 1 A_rp[r+1], 2 prods[r] / C_rp[r], 3 C_rp[r+1],
+  // 4 colmin[r], 5 colmax[r] (one round trip instead of six dependent loads)
+  auto fetch = [&](int64_t e, int32_t& row, int64_t& mv) {
+    row = -1;
+    mv = 0;
+    if (e < n) {
+      row = p.rows ? p.rows[e] : (int32_t)e;
+      if (lane == 0) mv = p.A_rp[row];
+      else if (lane == 1) mv = p.A_rp[row + 1];
+      else if (lane == 2) mv = PASS == 0 ? p.prods[row] : p.C_rp[row];
+      else if (lane == 3 && PASS == 1) mv = p.C_rp[row + 1];
+      else if (lane == 4) mv = p.colmin[row];
+      else if (lane == 5) mv = p.colmax[row];
+    }
+  };
+  // rows are claimed kWarpRowChunk at a time (one same-address atomic per chunk: per-row
+  // claims serialise at ~2-3 G/s in L2), the next chunk one chunk ahead
+  unsigned long long e = 0, cend = 0, nxt = 0;
+  if (lane == 0) {
+    e = atomicAdd(counter, (unsigned long long)kWarpRowChunk);
+    nxt = atomicAdd(counter, (unsigned long long)kWarpRowChunk);
+  }
+  e = __shfl_sync(0xffffffffu, e, 0);
+  nxt = __shfl_sync(0xffffffffu, nxt, 0);
+  cend = e + kWarpRowChunk;
+  int32_t row;
+  int64_t mv;
+  fetch((int64_t)e, row, mv);
+  while ((int64_t)e < n) {
+    unsigned long long en = e + 1;
+    if (en == cend) {                                     // chunk done: move to the claimed one
+      en = nxt;
+      cend = nxt + kWarpRowChunk;
+      if (lane == 0 && (int64_t)nxt < n) nxt = atomicAdd(counter, (unsigned long long)kWarpRowChunk);
+      nxt = __shfl_sync(0xffffffffu, nxt, 0);
+    }
+    const int64_t a0 = __shfl_sync(0xffffffffu, mv, 0);
+    const int alen = (int)(__shfl_sync(0xffffffffu, mv, 1) - a0);
+    const int64_t m2 = __shfl_sync(0xffffffffu, mv, 2);
+    const int64_t m3 = __shfl_sync(0xffffffffu, mv, 3);
+    const int32_t cmn = (int32_t)__shfl_sync(0xffffffffu, mv, 4);
+    const int32_t cmx = (int32_t)__shfl_sync(0xffffffffu, mv, 5);
+    const int32_t cur = row;
+    const int64_t need = PASS == 0 ? m2 : m3 - m2;       // products (symbolic) / exact nnz (numeric)
+    // region: symbolic 1.5x products (66% fill), numeric 2x entries (50% fill), 32-slot multiples
+    const uint64_t want = PASS == 0 ? (uint64_t)need * 3 / 2 : (uint64_t)need * 2;
+    const uint64_t w32 = (want + 31) & ~(uint64_t)31;
+    const uint32_t S = (uint32_t)(w32 < 64 ? 64 : (w32 > cap ? cap : w32));
+    fetch((int64_t)en, row, mv);                          // next row's metadata in flight
+    const int c = warp_row<PASS, V>(p, rk, rv, S, a0, alen, cmn, cmx, (int32_t)(m3 - m2), m2);
+    if (PASS == 0 && lane == 0) p.cnt[cur] = c;
+    e = en;
   }
 }
 

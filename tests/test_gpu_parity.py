@@ -174,6 +174,8 @@ PATHS = [
     dict(fixed_group_size=32),
     dict(fixed_group_size=1024),
     dict(concurrent_streams=1),
+    dict(warp_rows=0),
+    dict(warp_rows=0, global_lb_symbolic=0, global_lb_numeric=0),
 ]
 
 
