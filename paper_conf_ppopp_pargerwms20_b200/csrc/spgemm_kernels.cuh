@@ -28,6 +28,7 @@ namespace speck {
 
 constexpr int kSmallSeg = 64;   // rows with <= this many C entries are ranked, not sorted
 constexpr int kPPL = 4;         // products per lane per chunk in the warp-per-row path
+constexpr int kStreamLen = 64;  // referenced B rows at least this long are streamed, not balanced
 
 struct BlockMeta {
   int32_t row[kMaxGroupRows];
@@ -141,7 +142,9 @@ __device__ __forceinline__ int warp_write_ordered(const uint32_t* rk, const V* r
         while (re < S && rk[re] != kEmptyKey) ++re;
       }
       int rank = 0;
-      for (uint32_t j = rs; j < re; ++j) rank += rk[j] < k;
+      uint32_t j = rs;
+      for (; j + 4 <= re; j += 4) rank += (rk[j] < k) + (rk[j + 1] < k) + (rk[j + 2] < k) + (rk[j + 3] < k);
+      for (; j < re; ++j) rank += rk[j] < k;
       const int64_t o = ob + before + written + __popc(occ & lt) - (int)(s - rs) + rank;
       C_col[o] = (int32_t)k;
       C_val[o] = rv[s];
@@ -152,10 +155,41 @@ __device__ __forceinline__ int warp_write_ordered(const uint32_t* rk, const V* r
   return written;
 }
 
+// Linear probing over 4-slot groups for the unordered maps (symbolic keys, numeric rows of
+// <= kSmallSeg entries): one 16-byte shared load examines a whole group, a key takes the
+// first empty slot of the first group with room, groups are visited in order from the home
+// group (so the probe sequence of a key is fixed and, slots only ever going EMPTY -> key,
+// a key is never inserted twice).  At C5's ~67% symbolic load the scalar probe loop was half
+// of the symbolic kernel's instructions; groups cut the iterations ~4x.  keys must be 16-byte
+// aligned; only the first S & ~3 slots are used.
+__device__ __forceinline__ uint32_t probe_insert_grp(uint32_t* keys, uint32_t S, uint32_t key, bool* is_new) {
+  const uint32_t S4 = S & ~3u;
+  uint32_t g = hash_slot(key, S4) & ~3u;
+  while (true) {
+    uint4 q;
+    asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];"
+                 : "=r"(q.x), "=r"(q.y), "=r"(q.z), "=r"(q.w)
+                 : "r"((uint32_t)__cvta_generic_to_shared(keys + g)));
+    if (q.x == key) { *is_new = false; return g; }
+    if (q.y == key) { *is_new = false; return g + 1; }
+    if (q.z == key) { *is_new = false; return g + 2; }
+    if (q.w == key) { *is_new = false; return g + 3; }
+    const int e = q.x == kEmptyKey ? 0 : q.y == kEmptyKey ? 1 : q.z == kEmptyKey ? 2 : q.w == kEmptyKey ? 3 : -1;
+    if (e >= 0) {
+      const uint32_t old = atomicCAS(&keys[g + e], kEmptyKey, key);
+      if (old == kEmptyKey) { *is_new = true; return g + e; }
+      if (old == key) { *is_new = false; return g + e; }
+      continue;   // another key took the slot: re-read the group
+    }
+    g += 4;
+    if (g >= S4) g = 0;
+  }
+}
+
 // symbolic insert: true if the key was new
 __device__ __forceinline__ bool hash_insert_key(uint32_t* keys, uint32_t S, uint32_t col) {
   bool is_new;
-  probe_insert(keys, S, hash_slot(col, S), col, &is_new);
+  probe_insert_grp(keys, S, col, &is_new);
   return is_new;
 }
 
@@ -284,6 +318,33 @@ __device__ __forceinline__ void expand_row(const SpgemmArgs<V>& p, int64_t a0, i
       rng(f, p.B_rp[kc], p.B_rp[kc + 1], s, e);
       bst = s;
       blen = (int)(e - s);
+    }
+    // symbolic: long referenced B rows (>= kStreamLen products) are streamed by the warp
+    // directly — contiguous, coalesced loads, no owner search; the balanced expansion below
+    // takes the short ones (C3 symbolic 130 -> 83 ms).  The numeric pass keeps the balanced
+    // expansion for every row: a second inlined copy of its larger insert code cost more in
+    // instruction-cache misses than the search it saves (C5 numeric 429 -> 490 ms).
+    if (PASS == 0) {
+      const uint32_t lm = __ballot_sync(0xffffffffu, blen >= kStreamLen);
+      for (uint32_t rem = lm; rem; rem &= rem - 1) {
+        const int o = __ffs(rem) - 1;
+        const int64_t s0 = __shfl_sync(0xffffffffu, bst, o);
+        const int L = __shfl_sync(0xffffffffu, blen, o);
+        for (int q0 = c_first * CH; q0 < L; q0 += c_step * CH) {
+          uint32_t c[kPPL];
+#pragma unroll
+          for (int i = 0; i < kPPL; ++i) {
+            const int q = q0 + 32 * i + lane;
+            c[i] = q < L ? (uint32_t)p.B_col[s0 + q] : (0x80000000u | (uint32_t)lane);
+          }
+#pragma unroll
+          for (int i = 0; i < kPPL; ++i) {
+            if (q0 + 32 * i >= L) continue;   // warp-uniform
+            ins(c[i], V(0), q0 + 32 * i + lane < L);
+          }
+        }
+      }
+      if (blen >= kStreamLen) blen = 0;
     }
     const int incl = warp_incl_scan(blen);
     const int excl = incl - blen;
@@ -548,8 +609,9 @@ __device__ __forceinline__ int warp_row(const SpgemmArgs<V>& p, uint32_t* rk, V*
       const uint32_t peers = __match_any_sync(0xffffffffu, col);
       const uint32_t lt = (1u << lane_id()) - 1u;
       uint32_t s = 0;
-      if (act && !(peers & lt))
+      if (act && !(peers & lt)) {
         s = probe_insert_mono(rk, S, ordered ? mono_slot(col, mlo, mmult) : hash_slot(col, S), col, &wrapped);
+      }
       s = __shfl_sync(0xffffffffu, s, __ffs(peers) - 1);   // the key's slot, from its first lane
       const int rank = __popc(peers & lt);
       const int maxg = (int)__reduce_max_sync(0xffffffffu, (unsigned)__popc(peers));
@@ -639,7 +701,10 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
       const int64_t need = PASS == 0 ? pr : c;
       const int64_t need_tot = PASS == 0 ? tot_p : tot_c;
       uint32_t rsz = 0;
-      if (l < nr) rsz = nr == 1 ? cap : (need_tot > 0 ? (uint32_t)((uint64_t)cap * (uint64_t)need / (uint64_t)need_tot) : 0u);
+      // (multiples of 4 slots so 4-slot probe groups stay 16-byte aligned: 4 + a share of the rest)
+      if (l < nr)
+        rsz = nr == 1 ? cap
+                      : 4u + (need_tot > 0 ? (uint32_t)((uint64_t)(cap - 4u * nr) * (uint64_t)need / (uint64_t)need_tot) & ~3u : 0u);
       const uint32_t rinc = warp_incl_scan(rsz);
       const bool any_small = __any_sync(0xffffffffu, l < nr && c <= kSmallSeg);
       if (l < nr) {
