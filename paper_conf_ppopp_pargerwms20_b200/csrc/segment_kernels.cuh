@@ -63,7 +63,14 @@ struct SegPlanArgs {
   int64_t dense_window;    // columns of one dense window of the largest configuration
   int64_t map_slots;       // slots of the largest numeric hash map
   int prefer_parallel;     // few long rows: always split (parallelism across SMs)
+  int64_t bitmap_cols;     // >0: rows whose column range fits are done by k_long_bitmap (no segments)
 };
+
+// Long rows whose column range fits the shared-memory bitmap of k_long_bitmap.
+__device__ __forceinline__ bool bitmap_row(const SegPlanArgs& a, int32_t row) {
+  if (a.bitmap_cols <= 0) return false;
+  return (int64_t)a.colmax[row] + 1 - (a.colmin[row] & ~31) <= a.bitmap_cols;
+}
 
 // One "windows" job or column segments for a long row: estimated per-row overheads (the
 // products themselves cost the same either way).  Windows: per window, clear + scan the dense
@@ -91,7 +98,7 @@ __global__ void k_seg_count(SegPlanArgs a, int64_t* __restrict__ nseg) {
   const int32_t row = a.cand[e];
   const int64_t cnt = a.C_rp[row + 1] - a.C_rp[row];
   int64_t n = 0;
-  if (cnt > a.limit) {
+  if (cnt > a.limit && !bitmap_row(a, row)) {
     if (use_windows(a, row, cnt, a.map_slots)) {
       n = 1;
     } else {
@@ -109,7 +116,7 @@ __global__ void k_seg_emit(SegPlanArgs a, const int64_t* __restrict__ seg_off, S
   const int32_t row = a.cand[e];
   const int64_t c0 = a.C_rp[row];
   const int64_t cnt = a.C_rp[row + 1] - c0;
-  if (cnt <= a.limit) return;
+  if (cnt <= a.limit || bitmap_row(a, row)) return;
   const int32_t lo = a.colmin[row], hi = a.colmax[row];
   int64_t o = seg_off[e];
   if (use_windows(a, row, cnt, a.map_slots)) {
@@ -233,6 +240,106 @@ __global__ void __launch_bounds__(kCfgThreads[kSegCfg], 1024 / kCfgThreads[kSegC
       }
     }
   }
+}
+
+
+// ------------------------------------------------------------------------------------
+// Long rows by bitmap + rank (B200 design for rows beyond the largest hash map whose column
+// range fits a shared-memory bitmap; C3's ~175k long rows): one CTA of 1024 threads per row.
+//   1. structure: every product sets its column's bit (the symbolic pass's dense bitmap,
+//      P:1064-1084, recomputed: nothing survives between analyze and spgemm);
+//   2. one block scan gives every 32-bit word its exclusive prefix = the output position of
+//      its first entry; C.col is written in order from the bitmap (sorted by construction)
+//      and the row's C.val range is zeroed;
+//   3. values: every product's position is prefix[word] + popc(lower bits of its word), and
+//      a·b is added there with a global atomic (the row's C range stays in L2).
+// No column segments, no binary searches in B rows, no hash probing and no sort.  Columns are
+// relative to lo = colmin & ~31; smem: bits (4 B/word) + per-word prefix within its 32-word
+// group (uint16) + per-group prefix (int32).
+// ------------------------------------------------------------------------------------
+constexpr int kBitmapThreads = 1024;
+// 196 B of shared memory per 32-word group (128 bits + 4 prefix + 64 word prefixes)
+constexpr int64_t kBitmapMaxCols = (int64_t)(kCfgMapBytes[kNumCfg - 1] / 196) * 1024;
+
+template <typename V>
+__global__ void __launch_bounds__(kBitmapThreads, 1) k_long_bitmap(SpgemmArgs<V> p, SegPlanArgs a) {
+  constexpr int T = kBitmapThreads, NW = T / 32;
+  extern __shared__ __align__(16) unsigned char smem[];
+  __shared__ int64_t part[NW + 1];
+  const int32_t row = a.cand[blockIdx.x];
+  const int64_t ob = a.C_rp[row], cnt = a.C_rp[row + 1] - ob;
+  if (cnt <= a.limit || !bitmap_row(a, row)) return;
+  const int tid = threadIdx.x, lane = lane_id(), wp = warp_id();
+  const uint32_t lo = (uint32_t)a.colmin[row] & ~31u;
+  const int W = (int)(((int64_t)a.colmax[row] + 1 - lo + 31) / 32);
+  const int G = (W + 31) / 32;                                   // 32-word groups
+  uint32_t* bits = reinterpret_cast<uint32_t*>(smem);
+  int32_t* gpre = reinterpret_cast<int32_t*>(smem + (size_t)G * 128);       // after 32*G words
+  uint16_t* wpre = reinterpret_cast<uint16_t*>(smem + (size_t)G * 128 + (size_t)G * 4);
+  const int64_t a0 = p.A_rp[row];
+  const int alen = (int)(p.A_rp[row + 1] - a0);
+  for (int i = tid; i < G * 32; i += T) bits[i] = 0u;
+  __syncthreads();
+  // 1. structure
+  expand_row<0, V>(p, a0, alen, wp, NW, [&](uint32_t col, V, bool act) {
+    if (act) {
+      const uint32_t c = col - lo;
+      atomicOr(&bits[c >> 5], 1u << (c & 31));
+    }
+  });
+  __syncthreads();
+  // 2. prefixes: warp w owns groups [w*GW, (w+1)*GW); lane i holds word i of a group
+  const int GW = (G + NW - 1) / NW;
+  const int g0 = min(G, wp * GW), g1 = min(G, g0 + GW);
+  int wc = 0;
+  for (int g = g0; g < g1; ++g) wc += __popc(bits[g * 32 + lane]);
+  wc = warp_sum(wc);
+  if (lane == 0) part[wp] = wc;
+  __syncthreads();
+  int run = 0;
+  for (int w = 0; w < wp; ++w) run += (int)part[w];
+  for (int g = g0; g < g1; ++g) {
+    const uint32_t word = bits[g * 32 + lane];
+    const int pc = __popc(word);
+    const int incl = warp_incl_scan(pc);
+    const int excl = incl - pc;
+    wpre[g * 32 + lane] = (uint16_t)excl;
+    if (lane == 0) gpre[g] = run;
+    // C.col of the group: sparse groups per lane (a lane's entries are consecutive and the
+    // group's entries span few sectors), dense groups one word at a time across the warp
+    const int mx = __reduce_max_sync(0xffffffffu, (unsigned)pc);
+    const uint32_t cbase = lo + (uint32_t)g * 1024u;
+    if (mx <= 8) {
+      uint32_t wv = word;
+      int o = run + excl;
+      while (wv) {
+        const int b = __ffs(wv) - 1;
+        wv &= wv - 1;
+        p.C_col[ob + o++] = (int32_t)(cbase + (uint32_t)lane * 32u + (uint32_t)b);
+      }
+    } else {
+      for (int j = 0; j < 32; ++j) {
+        const uint32_t wj = __shfl_sync(0xffffffffu, word, j);
+        if (!wj) continue;
+        const int oj = __shfl_sync(0xffffffffu, excl, j);
+        if ((wj >> lane) & 1u)
+          p.C_col[ob + run + oj + __popc(wj & ((1u << lane) - 1u))] = (int32_t)(cbase + (uint32_t)j * 32u + (uint32_t)lane);
+      }
+    }
+    run += __shfl_sync(0xffffffffu, incl, 31);
+  }
+  // zero the row's values (coalesced), then make the zeros visible to the block's atomics
+  for (int64_t i = tid; i < cnt; i += T) p.C_val[ob + i] = V(0);
+  __syncthreads();
+  // 3. values
+  V* cv = p.C_val + ob;
+  expand_row<1, V, true>(p, a0, alen, wp, NW, [&](uint32_t col, V v, bool act) {
+    if (act) {
+      const uint32_t c = col - lo, w = c >> 5;
+      const int r = gpre[w >> 5] + (int)wpre[w] + __popc(bits[w] & ((1u << (c & 31)) - 1u));
+      atomicAdd(cv + r, v);
+    }
+  });
 }
 
 }  // namespace speck

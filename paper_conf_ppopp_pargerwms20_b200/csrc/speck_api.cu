@@ -62,6 +62,7 @@ struct speck_handle_s {
   // long-row segments
   int64_t opt_segments = 1;
   int64_t opt_warp_rows = 1;
+  int64_t opt_long_bitmap = 1;
   bool seg_enabled = false;
   int seg_shift = 15, nchunks = 0;
   int64_t long_thr = INT64_MAX, n_cand = 0, n_segs = 0, cand_start = 0;
@@ -205,6 +206,7 @@ speck_status_t set_smem_attrs(speck_handle_t h) {
     for (int pass = 0; pass < 2; ++pass)
       CK(cudaFuncSetAttribute(spgemm_fn<V>(c, pass), cudaFuncAttributeMaxDynamicSharedMemorySize, kCfgMapBytes[c]));
   CK(cudaFuncSetAttribute(k_segments<V>, cudaFuncAttributeMaxDynamicSharedMemorySize, kCfgMapBytes[kSegCfg]));
+  CK(cudaFuncSetAttribute(k_long_bitmap<V>, cudaFuncAttributeMaxDynamicSharedMemorySize, kCfgMapBytes[kNumCfg - 1]));
   CK(cudaFuncSetAttribute(k_warp_rows<0, V>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytes * (kWarpRowThreads / 32)));
   CK(cudaFuncSetAttribute(k_warp_rows<1, V>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytes * (kWarpRowThreads / 32)));
   return SPECK_OK;
@@ -348,6 +350,8 @@ SegPlanArgs seg_plan_args(speck_handle_t h, const int64_t* C_rp) {
   s.seg_limit = num_map_fill<V>(kSegCfg);
   // few candidates: split every long row so its work spreads over the SMs
   s.prefer_parallel = h->n_cand < 4 * (int64_t)h->num_sms ? 1 : 0;
+  // many long rows: one bitmap CTA per row whose column range fits (no column segments)
+  s.bitmap_cols = (h->opt_long_bitmap && !s.prefer_parallel) ? kBitmapMaxCols : 0;
   return s;
 }
 
@@ -396,6 +400,14 @@ speck_status_t run_pass(speck_handle_t h, int pass, int lb, const int64_t* cat_s
   if ((st = fork(h, s, ns))) return st;
   int si = 0;
   const int32_t* bins = static_cast<const int32_t*>(h->bins.p);
+  if (pass == 1 && h->seg_enabled && h->n_cand > 0) {
+    const SegPlanArgs sa = seg_plan_args<V>(h, a.C_rp);
+    if (sa.bitmap_cols > 0) {
+      k_long_bitmap<V><<<(unsigned)h->n_cand, kBitmapThreads, kCfgMapBytes[kNumCfg - 1], h->streams[si]>>>(a, sa);
+      CKL();
+      si = (si + 1) % ns;
+    }
+  }
   if (segs) {
     k_segments<V><<<(unsigned)h->n_segs, kCfgThreads[kSegCfg], kCfgMapBytes[kSegCfg], h->streams[si]>>>(
         a, static_cast<const Seg*>(h->segs.p));
@@ -821,6 +833,7 @@ speck_status_t speck_set_option(speck_handle_t h, int option, int64_t v) {
       h->opt_streams = v; break;
     case SPECK_OPT_SEGMENTS: h->opt_segments = v; break;
     case SPECK_OPT_WARP_ROWS: h->opt_warp_rows = v; break;
+    case SPECK_OPT_LONG_BITMAP: h->opt_long_bitmap = v; break;
     default: return fail(h, SPECK_ERR_INVALID_ARGUMENT, "unknown option %d", option);
   }
   return SPECK_OK;

@@ -294,7 +294,7 @@ struct FullRange {
   __device__ __forceinline__ void operator()(int, int64_t j0, int64_t j1, int64_t& s, int64_t& e) const { s = j0; e = j1; }
 };
 
-template <int PASS, typename V, typename Ins, typename Rng = FullRange>
+template <int PASS, typename V, bool STREAM = (PASS == 0), typename Ins, typename Rng = FullRange>
 __device__ __forceinline__ void expand_row(const SpgemmArgs<V>& p, int64_t a0, int alen, int wi, int nw, Ins&& ins,
                                            Rng rng = Rng()) {
   const int lane = lane_id();
@@ -319,28 +319,32 @@ __device__ __forceinline__ void expand_row(const SpgemmArgs<V>& p, int64_t a0, i
       bst = s;
       blen = (int)(e - s);
     }
-    // symbolic: long referenced B rows (>= kStreamLen products) are streamed by the warp
-    // directly — contiguous, coalesced loads, no owner search; the balanced expansion below
-    // takes the short ones (C3 symbolic 130 -> 83 ms).  The numeric pass keeps the balanced
-    // expansion for every row: a second inlined copy of its larger insert code cost more in
-    // instruction-cache misses than the search it saves (C5 numeric 429 -> 490 ms).
-    if (PASS == 0) {
+    // STREAM (symbolic, long-row bitmap kernel): long referenced B rows (>= kStreamLen
+    // products) are streamed by the warp directly — contiguous, coalesced loads, no owner
+    // search; the balanced expansion below takes the short ones (C3 symbolic 130 -> 83 ms).
+    // The hash-map numeric kernels keep the balanced expansion for every row: a second
+    // inlined copy of their larger insert code cost more in instruction-cache misses than the
+    // search it saves (C5 numeric 429 -> 490 ms).
+    if (STREAM) {
       const uint32_t lm = __ballot_sync(0xffffffffu, blen >= kStreamLen);
       for (uint32_t rem = lm; rem; rem &= rem - 1) {
         const int o = __ffs(rem) - 1;
         const int64_t s0 = __shfl_sync(0xffffffffu, bst, o);
         const int L = __shfl_sync(0xffffffffu, blen, o);
+        const V ao = PASS == 1 ? __shfl_sync(0xffffffffu, a, o) : V(0);
         for (int q0 = c_first * CH; q0 < L; q0 += c_step * CH) {
           uint32_t c[kPPL];
+          V bv[kPPL];
 #pragma unroll
           for (int i = 0; i < kPPL; ++i) {
             const int q = q0 + 32 * i + lane;
             c[i] = q < L ? (uint32_t)p.B_col[s0 + q] : (0x80000000u | (uint32_t)lane);
+            bv[i] = (PASS == 1 && q < L) ? ldv(p.B_val + s0 + q) : V(0);
           }
 #pragma unroll
           for (int i = 0; i < kPPL; ++i) {
             if (q0 + 32 * i >= L) continue;   // warp-uniform
-            ins(c[i], V(0), q0 + 32 * i + lane < L);
+            ins(c[i], ao * bv[i], q0 + 32 * i + lane < L);
           }
         }
       }

@@ -213,6 +213,29 @@ def test_long_rows(dev, segments, dt):
     assert_parity(A2, B2, C2)
 
 
+@pytest.mark.parametrize("long_bitmap", [1, 0])
+@pytest.mark.parametrize("dt", [torch.float32, torch.float64])
+def test_many_long_rows_bitmap(dev, long_bitmap, dt):
+    """>= 4 long rows per SM (C3-like): each long row of C is one bitmap + rank CTA when its
+    column range fits the shared-memory bitmap, else (and with long_bitmap=0) column segments.
+    700 rows x 24 B rows of 1000 random columns of 2^20 -> ~24k entries per row (> the largest
+    hash map); the last 100 rows reach columns up to 1.5M (range too wide: segments)."""
+    import numpy as _np
+    rng = _np.random.default_rng(7)
+    nb, lb = 3000, 1000
+    ncols = np.where(np.arange(nb) < 2800, 1 << 20, 1_500_000)
+    cols = np.stack([np.sort(rng.choice(int(n), size=lb, replace=False)) for n in ncols])
+    B = W.csr_from_coo(nb, 1_500_000, torch.arange(nb).repeat_interleave(lb), torch.tensor(cols.reshape(-1)), None,
+                       dtype=dt, seed=8)
+    ar = np.repeat(np.arange(700), 24)
+    ac = np.concatenate([np.sort(rng.choice(2800, 24, replace=False)) if i < 600
+                         else np.sort(rng.choice(nb, 24, replace=False)) for i in range(700)])
+    A = W.csr_from_coo(700, nb, torch.tensor(ar), torch.tensor(ac), None, dtype=dt, seed=9)
+    C, st = gpu_spgemm(A, B, long_bitmap=long_bitmap)
+    assert st["rows_per_bin_numeric"][7] >= 600
+    assert_parity(A, B, C)
+
+
 def test_fig5_dense_window_of_three(dev):
     """Fig. 5: one row, 6 columns, window 3, products at c0,c2,c4,c4,c5 -> c0=1 c2=1 c4=2 c5=1."""
     kv, _ = golden("fig5_dense.txt")
