@@ -294,9 +294,19 @@ struct FullRange {
   __device__ __forceinline__ void operator()(int, int64_t j0, int64_t j1, int64_t& s, int64_t& e) const { s = j0; e = j1; }
 };
 
+// First batch of a row loaded ahead of time (k_warp_rows pipelines it one row ahead): lane f
+// holds B row start/length and a of the row's f-th NZ.
+template <typename V>
+struct PreBatch {
+  int64_t bst = 0;
+  int blen = 0;
+  V a = V(0);
+  bool valid = false;
+};
+
 template <int PASS, typename V, bool STREAM = (PASS == 0), typename Ins, typename Rng = FullRange>
 __device__ __forceinline__ void expand_row(const SpgemmArgs<V>& p, int64_t a0, int alen, int wi, int nw, Ins&& ins,
-                                           Rng rng = Rng()) {
+                                           Rng rng = Rng(), const PreBatch<V>* pre = nullptr) {
   const int lane = lane_id();
   const int nb = (alen + 31) >> 5;
   constexpr int CH = 32 * kPPL;
@@ -311,7 +321,11 @@ __device__ __forceinline__ void expand_row(const SpgemmArgs<V>& p, int64_t a0, i
     int64_t bst = 0;
     int blen = 0;
     V a = V(0);
-    if (f < alen) {
+    if (pre && b == 0 && pre->valid) {
+      bst = pre->bst;
+      blen = pre->blen;
+      a = pre->a;
+    } else if (f < alen) {
       const int32_t kc = p.A_col[a0 + f];
       if (PASS == 1) a = ldv(p.A_val + a0 + f);
       int64_t s, e;
@@ -593,7 +607,8 @@ __device__ __noinline__ void block_sorted_write(uint32_t* keys, V* vals, uint32_
 // (ordered map for rows > kSmallSeg entries, else rank counting).  Returns the symbolic count.
 template <int PASS, typename V>
 __device__ __forceinline__ int warp_row(const SpgemmArgs<V>& p, uint32_t* rk, V* rv, uint32_t S, int64_t a0, int alen,
-                                        int32_t cmin, int32_t cmax, int32_t cnt, int64_t cbase) {
+                                        int32_t cmin, int32_t cmax, int32_t cnt, int64_t cbase,
+                                        const PreBatch<V>* pre = nullptr) {
   const int lane = lane_id();
   for (uint32_t i = lane; i < S; i += 32) {
     rk[i] = kEmptyKey;
@@ -606,7 +621,8 @@ __device__ __forceinline__ int warp_row(const SpgemmArgs<V>& p, uint32_t* rk, V*
   // short rows keep the scrambled hash (robust to clustered columns) and rank counting
   const bool ordered = PASS == 1 && cnt > kSmallSeg;
   int newc = 0, wrapped = 0;
-  expand_row<PASS, V>(p, a0, alen, 0, 1, [&](uint32_t col, V v, bool act) {
+  expand_row<PASS, V>(
+      p, a0, alen, 0, 1, [&](uint32_t col, V v, bool act) {
     if (PASS == 0) {
       if (act) newc += hash_insert_key(rk, S, col);
     } else {
@@ -977,17 +993,44 @@ __global__ void __launch_bounds__(kWarpRowThreads, kWarpRowCtasPerSM)
   e = __shfl_sync(0xffffffffu, e, 0);
   nxt = __shfl_sync(0xffffffffu, nxt, 0);
   cend = e + kWarpRowChunk;
-  int32_t row;
-  int64_t mv;
-  fetch((int64_t)e, row, mv);
-  while ((int64_t)e < n) {
-    unsigned long long en = e + 1;
-    if (en == cend) {                                     // chunk done: move to the claimed one
-      en = nxt;
+  // the first batch of a row (A col/val -> B row start/length, two dependent round trips) is
+  // loaded one row ahead, the metadata two rows ahead: a row's only exposed latency is its
+  // B gathers
+  auto fetch_batch = [&](int64_t a0, int alen, PreBatch<V>& bt) {
+    bt.valid = true;
+    bt.bst = 0;
+    bt.blen = 0;
+    bt.a = V(0);
+    if (lane < alen) {
+      const int32_t kc = p.A_col[a0 + lane];
+      if (PASS == 1) bt.a = ldv(p.A_val + a0 + lane);
+      bt.bst = p.B_rp[kc];
+      bt.blen = (int)(p.B_rp[kc + 1] - bt.bst);
+    }
+  };
+  auto next_index = [&](unsigned long long x) {
+    unsigned long long y = x + 1;
+    if (y == cend) {                                      // chunk done: move to the claimed one
+      y = nxt;
       cend = nxt + kWarpRowChunk;
       if (lane == 0 && (int64_t)nxt < n) nxt = atomicAdd(counter, (unsigned long long)kWarpRowChunk);
       nxt = __shfl_sync(0xffffffffu, nxt, 0);
     }
+    return y;
+  };
+  int32_t row;
+  int64_t mv;
+  fetch((int64_t)e, row, mv);
+  PreBatch<V> bt;
+  {
+    const int64_t a0 = __shfl_sync(0xffffffffu, mv, 0);
+    fetch_batch(a0, (int)(__shfl_sync(0xffffffffu, mv, 1) - a0), bt);
+  }
+  unsigned long long en = next_index(e);
+  int32_t rown;
+  int64_t mvn;
+  fetch((int64_t)en, rown, mvn);
+  while ((int64_t)e < n) {
     const int64_t a0 = __shfl_sync(0xffffffffu, mv, 0);
     const int alen = (int)(__shfl_sync(0xffffffffu, mv, 1) - a0);
     const int64_t m2 = __shfl_sync(0xffffffffu, mv, 2);
@@ -1000,10 +1043,20 @@ __global__ void __launch_bounds__(kWarpRowThreads, kWarpRowCtasPerSM)
     const uint64_t want = PASS == 0 ? (uint64_t)need * 3 / 2 : (uint64_t)need * 2;
     const uint64_t w32 = (want + 31) & ~(uint64_t)31;
     const uint32_t S = (uint32_t)(w32 < 64 ? 64 : (w32 > cap ? cap : w32));
-    fetch((int64_t)en, row, mv);                          // next row's metadata in flight
-    const int c = warp_row<PASS, V>(p, rk, rv, S, a0, alen, cmn, cmx, (int32_t)(m3 - m2), m2);
+    const PreBatch<V> bcur = bt;
+    // pipeline: next row's batch, the row after next's metadata
+    const unsigned long long enn = (int64_t)en < n ? next_index(en) : en;
+    if ((int64_t)en < n) {
+      const int64_t a0n = __shfl_sync(0xffffffffu, mvn, 0);
+      fetch_batch(a0n, (int)(__shfl_sync(0xffffffffu, mvn, 1) - a0n), bt);
+    }
+    row = rown;
+    mv = mvn;
+    fetch((int64_t)enn, rown, mvn);
+    const int c = warp_row<PASS, V>(p, rk, rv, S, a0, alen, cmn, cmx, (int32_t)(m3 - m2), m2, &bcur);
     if (PASS == 0 && lane == 0) p.cnt[cur] = c;
     e = en;
+    en = enn;
   }
 }
 
