@@ -253,7 +253,9 @@ __global__ void __launch_bounds__(kCfgThreads[kSegCfg], 1024 / kCfgThreads[kSegC
 //      and the row's C.val range is zeroed;
 //   3. values: every product's position is prefix[word] + popc(lower bits of its word), and
 //      a·b is added there with a global atomic (the row's C range stays in L2).
-// No column segments, no binary searches in B rows, no hash probing and no sort.  Columns are
+// No column segments, no binary searches in B rows, no hash probing and no sort.  Both passes
+// rotate product chunks over all 32 warps (expand_row ALL): a hub row of B referenced by the
+// row is streamed by every warp, not by the one warp whose batch holds it.  Columns are
 // relative to lo = colmin & ~31; smem: bits (4 B/word) + per-word prefix within its 32-word
 // group (uint16) + per-group prefix (int32).
 // ------------------------------------------------------------------------------------
@@ -281,7 +283,7 @@ __global__ void __launch_bounds__(kBitmapThreads, 1) k_long_bitmap(SpgemmArgs<V>
   for (int i = tid; i < G * 32; i += T) bits[i] = 0u;
   __syncthreads();
   // 1. structure
-  expand_row<0, V>(p, a0, alen, wp, NW, [&](uint32_t col, V, bool act) {
+  expand_row<0, V, true, true>(p, a0, alen, wp, NW, [&](uint32_t col, V, bool act) {
     if (act) {
       const uint32_t c = col - lo;
       atomicOr(&bits[c >> 5], 1u << (c & 31));
@@ -333,7 +335,7 @@ __global__ void __launch_bounds__(kBitmapThreads, 1) k_long_bitmap(SpgemmArgs<V>
   __syncthreads();
   // 3. values
   V* cv = p.C_val + ob;
-  expand_row<1, V, true>(p, a0, alen, wp, NW, [&](uint32_t col, V v, bool act) {
+  expand_row<1, V, true, true>(p, a0, alen, wp, NW, [&](uint32_t col, V v, bool act) {
     if (act) {
       const uint32_t c = col - lo, w = c >> 5;
       const int r = gpre[w >> 5] + (int)wpre[w] + __popc(bits[w] & ((1u << (c & 31)) - 1u));

@@ -304,7 +304,15 @@ struct PreBatch {
   bool valid = false;
 };
 
-template <int PASS, typename V, bool STREAM = (PASS == 0), typename Ins, typename Rng = FullRange>
+//
+// ALL = true (single-row blocks): every warp reads every batch (its 32 A entries and B row
+// bounds, L1-resident after the first warp) and the batch's product chunks go round-robin over
+// all nw warps, continuing the rotation across batches and streamed rows, so every warp ends
+// within one chunk of the others — no warp waits at the block barrier for a batch holding a
+// hub row of B (ncu, C5: 22-50% of the stall samples of the single-row kernels were that
+// barrier with batches assigned round-robin).  Rng must then be pure (evaluated by every warp)
+// or write the same value from every warp.
+template <int PASS, typename V, bool STREAM = (PASS == 0), bool ALL = false, typename Ins, typename Rng = FullRange>
 __device__ __forceinline__ void expand_row(const SpgemmArgs<V>& p, int64_t a0, int alen, int wi, int nw, Ins&& ins,
                                            Rng rng = Rng(), const PreBatch<V>* pre = nullptr) {
   const int lane = lane_id();
@@ -312,10 +320,17 @@ __device__ __forceinline__ void expand_row(const SpgemmArgs<V>& p, int64_t a0, i
   constexpr int CH = 32 * kPPL;
   // fewer batches than warps: G = nw/nb warps per batch, splitting its product chunks;
   // otherwise batches go round-robin and a warp takes all chunks of its batch
-  const int G = nb >= nw ? 1 : nw / nb;
+  const int G = ALL ? nw : (nb >= nw ? 1 : nw / nb);
   const bool share = G > 1;
-  const int b_first = share ? wi / G : wi, b_step = share ? nb : nw;   // share: one batch per warp group
-  const int c_first = share ? wi % G : 0, c_step = share ? G : 1;
+  const int b_first = ALL ? 0 : (share ? wi / G : wi), b_step = ALL ? 1 : (share ? nb : nw);
+  int c_first = ALL ? 0 : (share ? wi % G : 0);
+  const int c_step = share ? G : 1;
+  int rot = 0;   // ALL: warp taking the next chunk (warp-uniform, identical in every warp)
+  auto my_first = [&](int nsub) {   // ALL: first chunk of this warp among nsub, then advance the rotation
+    const int j0 = (wi - rot + nw) % nw;
+    rot = (rot + nsub) % nw;
+    return j0;
+  };
   for (int b = b_first; b < nb; b += b_step) {
     const int f = b * 32 + lane;
     int64_t bst = 0;
@@ -346,6 +361,7 @@ __device__ __forceinline__ void expand_row(const SpgemmArgs<V>& p, int64_t a0, i
         const int64_t s0 = __shfl_sync(0xffffffffu, bst, o);
         const int L = __shfl_sync(0xffffffffu, blen, o);
         const V ao = PASS == 1 ? __shfl_sync(0xffffffffu, a, o) : V(0);
+        if (ALL) c_first = my_first((L + CH - 1) / CH);
         for (int q0 = c_first * CH; q0 < L; q0 += c_step * CH) {
           uint32_t c[kPPL];
           V bv[kPPL];
@@ -395,6 +411,7 @@ __device__ __forceinline__ void expand_row(const SpgemmArgs<V>& p, int64_t a0, i
     uint32_t ca[kPPL];
     V va[kPPL];
     int oa[kPPL];
+    if (ALL) c_first = my_first((Pb + CH - 1) / CH);
     for (int p0 = c_first * CH; p0 < Pb; p0 += c_step * CH) {
       gather(p0, ca, va, oa);
 #pragma unroll
@@ -722,9 +739,18 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
       const int64_t need_tot = PASS == 0 ? tot_p : tot_c;
       uint32_t rsz = 0;
       // (multiples of 4 slots so 4-slot probe groups stay 16-byte aligned: 4 + a share of the rest)
-      if (l < nr)
-        rsz = nr == 1 ? cap
-                      : 4u + (need_tot > 0 ? (uint32_t)((uint64_t)(cap - 4u * nr) * (uint64_t)need / (uint64_t)need_tot) & ~3u : 0u);
+      // A single row gets a region sized to it (symbolic 1.5x products = 66% fill, numeric 2x
+      // entries = 50%), so clearing and the write-out scan touch only the slots the row can use
+      // (C5: the write-out scan of the full map was over half of the numeric instructions).
+      if (l < nr) {
+        if (nr == 1) {
+          const uint64_t want = PASS == 0 ? (uint64_t)need * 3 / 2 : (uint64_t)need * 2;
+          const uint64_t w32 = (want + 31) & ~(uint64_t)31;
+          rsz = (uint32_t)(w32 < 64 ? 64 : (w32 > cap ? cap : w32));
+        } else {
+          rsz = 4u + (need_tot > 0 ? (uint32_t)((uint64_t)(cap - 4u * nr) * (uint64_t)need / (uint64_t)need_tot) & ~3u : 0u);
+        }
+      }
       const uint32_t rinc = warp_incl_scan(rsz);
       const bool any_small = __any_sync(0xffffffffu, l < nr && c <= kSmallSeg);
       if (l < nr) {
@@ -814,7 +840,7 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
         const uint64_t mmult = mono_mult((uint32_t)(bm.rhi[r] - bm.rlo[r] + 1), S);
         const bool ordered = bm.ordered;
         int newc = 0, wrapped = 0;
-        expand_row<PASS, V>(p, bm.astart[r], (int)(bm.aoff[r + 1] - bm.aoff[r]), warp_id(), NW,
+        expand_row<PASS, V, PASS == 0, true>(p, bm.astart[r], (int)(bm.aoff[r + 1] - bm.aoff[r]), warp_id(), NW,
                             [&](uint32_t col, V v, bool act) {
                               if (PASS == 0) {
                                 if (act) newc += hash_insert_key(rk, S, col);
@@ -916,7 +942,7 @@ __device__ __noinline__ void dense_row(const SpgemmArgs<V>& p, BlockMeta& bm, in
         __syncthreads();
         // expand-balanced accumulation of the products falling into this window
         auto ins = [&](uint32_t col, V v, bool act) { dense_insert<PASS, V>(bits, dvals, (uint32_t)wlo, col, v, act); };
-        if (nwin == 1) expand_row<PASS, V>(p, astart, (int)nnzA, warp_id(), NW, ins);
+        if (nwin == 1) expand_row<PASS, V, PASS == 0, true>(p, astart, (int)nnzA, warp_id(), NW, ins);
         else expand_row<PASS, V>(p, astart, (int)nnzA, warp_id(), NW, ins, WindowRange{res, res_next, p.B_col, (uint32_t)whi});
         __syncthreads();
         { int32_t* t_ = res; res = res_next; res_next = t_; }
