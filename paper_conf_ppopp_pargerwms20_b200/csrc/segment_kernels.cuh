@@ -183,7 +183,7 @@ __global__ void __launch_bounds__(kCfgThreads[kSegCfg], 1024 / kCfgThreads[kSegC
     uint32_t* keys = reinterpret_cast<uint32_t*>(smem);
     V* vals = reinterpret_cast<V*>(smem + num_val_offset<V>(CFG));
     const uint32_t S = num_map_cap<V>(CFG);
-    const uint64_t mmult = mono_mult(range, S);
+    const uint64_t mmult = bkt_mult(range, S);
     for (uint32_t i = tid; i < S; i += T) { keys[i] = kEmptyKey; vals[i] = V(0); }
     if (tid == 0) s_wrap = 0;
     __syncthreads();
@@ -192,7 +192,7 @@ __global__ void __launch_bounds__(kCfgThreads[kSegCfg], 1024 / kCfgThreads[kSegC
         p, a0, alen, warp_id(), NW,
         [&](uint32_t col, V v, bool act) {
           uint32_t s = 0;
-          if (act) s = probe_insert_mono(keys, S, mono_slot(col, lo, mmult), col, &wrapped);
+          if (act) s = probe_insert_bkt(keys, S >> 3, bkt_home(col, lo, mmult), col, &wrapped);
           bool leader;
           const V sum = warp_key_sum(col, v, leader);
           if (act && leader) atomicAdd(&vals[s], sum);

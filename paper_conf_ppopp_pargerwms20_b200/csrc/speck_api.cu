@@ -207,8 +207,10 @@ speck_status_t set_smem_attrs(speck_handle_t h) {
       CK(cudaFuncSetAttribute(spgemm_fn<V>(c, pass), cudaFuncAttributeMaxDynamicSharedMemorySize, kCfgMapBytes[c]));
   CK(cudaFuncSetAttribute(k_segments<V>, cudaFuncAttributeMaxDynamicSharedMemorySize, kCfgMapBytes[kSegCfg]));
   CK(cudaFuncSetAttribute(k_long_bitmap<V>, cudaFuncAttributeMaxDynamicSharedMemorySize, kCfgMapBytes[kNumCfg - 1]));
-  CK(cudaFuncSetAttribute(k_warp_rows<0, V>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytes * (kWarpRowThreads / 32)));
-  CK(cudaFuncSetAttribute(k_warp_rows<1, V>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytes * (kWarpRowThreads / 32)));
+  CK(cudaFuncSetAttribute(k_warp_rows<0, V, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytes * (kWarpRowThreads / 32)));
+  CK(cudaFuncSetAttribute(k_warp_rows<1, V, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytes * (kWarpRowThreads / 32)));
+  CK(cudaFuncSetAttribute(k_warp_rows<1, V, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytes * (kWarpRowThreads / 32)));
+  CK(cudaFuncSetAttribute(k_warp_rows<1, V, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytes * (kWarpRowThreads / 32)));
   return SPECK_OK;
 }
 
@@ -245,15 +247,19 @@ int64_t warp_row_fill(speck_handle_t h, int pass) {
 }
 
 // Small-row kernel: persistent CTAs of 8 warps pulling rows from a counter (zeroed here).
+// mode (numeric): 0 any row, 1 rows of <= kTinyCnt entries, 2 larger rows (k_warp_rows MODE).
 template <typename V>
-speck_status_t launch_warp_rows(speck_handle_t h, int pass, const SpgemmArgs<V>& a, cudaStream_t s) {
+speck_status_t launch_warp_rows(speck_handle_t h, int pass, const SpgemmArgs<V>& a, cudaStream_t s, int mode = 0) {
   if (a.n_entries <= 0) return SPECK_OK;
-  unsigned long long* ctr = reinterpret_cast<unsigned long long*>(static_cast<char*>(h->small.p) + 1024 + 8 * pass);
+  unsigned long long* ctr =
+      reinterpret_cast<unsigned long long*>(static_cast<char*>(h->small.p) + 1024 + 8 * (pass == 0 ? 0 : 1 + mode));
   CK(cudaMemsetAsync(ctr, 0, 8, s));
   const int64_t grid = std::min<int64_t>((a.n_entries + 7) / 8, (int64_t)h->num_sms * kWarpRowCtasPerSM);
   const size_t smem = (size_t)kWarpRegionBytes * (kWarpRowThreads / 32);
-  if (pass == 0) k_warp_rows<0, V><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
-  else k_warp_rows<1, V><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
+  if (pass == 0) k_warp_rows<0, V, 0><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
+  else if (mode == 1) k_warp_rows<1, V, 1><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
+  else if (mode == 2) k_warp_rows<1, V, 2><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
+  else k_warp_rows<1, V, 0><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
   CKL();
   return SPECK_OK;
 }
@@ -263,6 +269,7 @@ BinParams make_bin_params(speck_handle_t h, int pass) {
   bp.pass = pass;
   bp.use_direct = h->opt_disable_direct ? 0 : 1;
   bp.long_thr = INT64_MAX;
+  bp.tiny_cap = (pass == 1 && h->opt_warp_rows) ? kTinyCnt : -1;
   for (int c = 0; c < kNumCfg; ++c) {
     if (pass == 0) bp.cap[c] = sym_map_fill(c);
     else bp.cap[c] = h->dtype == SPECK_F64 ? num_map_fill<double>(c) : num_map_fill<float>(c);
@@ -370,7 +377,8 @@ speck_status_t run_pass(speck_handle_t h, int pass, int lb, const int64_t* cat_s
       own.cap[c] = pass == 0 ? (int64_t)sym_map_fill(c) : (int64_t)num_map_fill<V>(c);
     a.rows = nullptr;
     a.n_entries = m;
-    if (h->opt_warp_rows && need_max <= warp_row_fill(h, pass)) return launch_warp_rows<V>(h, pass, a, s);
+    if (h->opt_warp_rows && need_max <= warp_row_fill(h, pass))
+      return launch_warp_rows<V>(h, pass, a, s, pass == 1 && need_max <= kTinyCnt ? 1 : 0);
     int cfg = -1, R = 1;
     for (int c = 0; c < kNumCfg; ++c)
       if (need_max * kMaxGroupRows <= own.cap[c]) { cfg = c; R = kMaxGroupRows; break; }
@@ -423,7 +431,7 @@ speck_status_t run_pass(speck_handle_t h, int pass, int lb, const int64_t* cat_s
     b.rows = bins + cat_start[cat];
     b.n_entries = n;
     if (c == 0 && h->opt_warp_rows) {
-      st = launch_warp_rows<V>(h, pass, b, h->streams[si]);
+      st = launch_warp_rows<V>(h, pass, b, h->streams[si], pass == 1 ? 2 : 0);
       if (st) return st;
       si = (si + 1) % ns;
       continue;
@@ -443,6 +451,14 @@ speck_status_t run_pass(speck_handle_t h, int pass, int lb, const int64_t* cat_s
       b.long_thr = h->long_thr;
     }
     st = launch_spgemm<V>(h, c, pass, b, h->streams[si]);
+    if (st) return st;
+    si = (si + 1) % ns;
+  }
+  if (pass == 1 && cat_start[CAT_TINY + 1] > cat_start[CAT_TINY]) {
+    SpgemmArgs<V> b = a;
+    b.rows = bins + cat_start[CAT_TINY];
+    b.n_entries = cat_start[CAT_TINY + 1] - cat_start[CAT_TINY];
+    st = launch_warp_rows<V>(h, pass, b, h->streams[si], 1);
     if (st) return st;
     si = (si + 1) % ns;
   }
@@ -562,7 +578,7 @@ speck_status_t analyze_impl(speck_handle_t h, const speck_csr_t* A, const speck_
   h->st.max_row_products = (int64_t)hs.max_prods;
   h->st.rows_direct = (int64_t)hs.n_direct;
   h->st.rows_empty = (int64_t)hs.n_empty;
-  for (int c = 0; c < CAT_COUNT; ++c) h->st.rows_per_bin_symbolic[c] = sym_cat[c + 1] - sym_cat[c];
+  for (int c = 0; c < CAT_TINY; ++c) h->st.rows_per_bin_symbolic[c] = sym_cat[c + 1] - sym_cat[c];
   if ((st = timing_mark(h, 1, s))) return st;
 
   // resume scratch for multi-window dense rows (largest configuration, one CTA per SM)
@@ -639,7 +655,9 @@ speck_status_t analyze_impl(speck_handle_t h, const speck_csr_t* A, const speck_
   h->n_segs = (int64_t)h->h_pinned[2];
   h->st.segments = h->n_segs;
   for (int c = 0; c <= CAT_COUNT; ++c) h->num_cat_start[c] = (int64_t)h->h_pinned[16 + c];
-  for (int c = 0; c < CAT_COUNT; ++c) h->st.rows_per_bin_numeric[c] = h->num_cat_start[c + 1] - h->num_cat_start[c];
+  for (int c = 0; c < CAT_TINY; ++c) h->st.rows_per_bin_numeric[c] = h->num_cat_start[c + 1] - h->num_cat_start[c];
+  // the stats keep one smallest-configuration count (tiny rows included)
+  h->st.rows_per_bin_numeric[CAT_CFG0] += h->num_cat_start[CAT_TINY + 1] - h->num_cat_start[CAT_TINY];
   *nnz_c = h->nnz_c;
   h->st.nnz_c = h->nnz_c;
   if (h->opt_timing) {

@@ -42,8 +42,13 @@ enum Cat : int {
   CAT_DIRECT = 1, // single NZ in the row of A
   CAT_CFG0 = 2,   // CAT_CFG0 + j = configuration j (cfg0 bin = merged small rows)
   CAT_LONG = CAT_CFG0 + kNumCfg,  // numeric rows beyond the largest map: split into column segments
-  CAT_COUNT = CAT_LONG + 1
+  CAT_TINY = CAT_LONG + 1,        // numeric rows of the smallest bin with <= kTinyCnt entries (rank-counted)
+  CAT_COUNT = CAT_TINY + 1
 };
+// numeric rows with at most this many entries keep a scrambled hash and rank counting
+// (P:1130-1133); larger ones use the order-preserving map.  They get separate warp-row
+// kernels so each stays compact in the instruction cache.
+constexpr int kTinyCnt = 64;
 
 // Long rows (numeric nnz beyond the largest hash map) are split into column segments whose
 // exact sizes come from per-chunk counts recorded by the symbolic pass: chunks of 2^s
@@ -138,6 +143,7 @@ struct BinParams {
   int use_direct;           // route single-NZ rows to the direct path
   int64_t cap[kNumCfg];     // need thresholds: row goes to the smallest cfg with need <= cap[cfg]
   int64_t long_thr;         // numeric: rows with cnt > long_thr are split into segments
+  int64_t tiny_cap;         // numeric: smallest-bin rows with cnt <= tiny_cap go to CAT_TINY (-1: off)
 };
 
 __host__ __device__ inline int classify_row(int64_t nnza, int64_t prods, int64_t cnt, const BinParams& bp) {
@@ -146,6 +152,7 @@ __host__ __device__ inline int classify_row(int64_t nnza, int64_t prods, int64_t
   if (bp.pass == 1 && cnt > bp.long_thr) return CAT_LONG;
   int64_t need = bp.pass == 0 ? prods : cnt;
 #pragma unroll
+  if (bp.pass == 1 && need <= bp.tiny_cap && need <= bp.cap[0]) return CAT_TINY;
   for (int c = 0; c < kNumCfg - 1; ++c)
     if (need <= bp.cap[c]) return CAT_CFG0 + c;
   return CAT_CFG0 + kNumCfg - 1;

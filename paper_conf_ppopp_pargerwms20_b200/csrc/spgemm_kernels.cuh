@@ -26,7 +26,7 @@
 
 namespace speck {
 
-constexpr int kSmallSeg = 64;   // rows with <= this many C entries are ranked, not sorted
+constexpr int kSmallSeg = kTinyCnt;   // rows with <= this many C entries are ranked, not sorted
 constexpr int kPPL = 4;         // products per lane per chunk in the warp-per-row path
 constexpr int kStreamLen = 64;  // referenced B rows at least this long are streamed, not balanced
 
@@ -76,19 +76,48 @@ __device__ __forceinline__ uint32_t probe_insert(uint32_t* keys, uint32_t S, uin
   }
 }
 
-// Order-preserving home slot for the numeric maps: homes are monotone in the column over the
-// row's [colmin, colmax] and occupy the first 7/8 of the region, the rest absorbs probing
-// runs.  With linear probing and no wrap-around, every key sits in the run ("cluster") that
-// contains its home, and clusters appear in column order; an entry's position in the sorted
-// row is therefore (#occupied slots before its cluster) + (rank of its key inside the cluster).
-// home = floor((col - lo) * mult / 2^32) with mult = floor(sh * 2^32 / range), sh = 7/8 S:
-// monotone in col, < sh, and a multiply per product instead of a 64-bit division.
-__device__ __forceinline__ uint64_t mono_mult(uint32_t range, uint32_t S) {
-  const uint64_t sh = S - (S >> 3);
-  return range ? (sh << 32) / range : 0;
+// Order-preserving numeric maps: 8-slot buckets, the home bucket monotone in the column over
+// the row's [colmin, colmax] and covering the first 7/8 of the buckets (the rest absorbs
+// overflow).  A key takes the first empty slot of its home bucket, or of the next non-full
+// bucket; occupied slots of a bucket are always a prefix of it.  Hence every key sits in the
+// probing run (maximal occupied range) that contains its home, runs appear in column order, and
+// an entry's position in the sorted row is (#occupied slots before its run) + (rank of its key
+// in the run); a run that ends in a non-full bucket and starts after one is just that bucket
+// (warp_write_ordered's fast path ranks it with 7 shuffles).
+// home = floor((col - lo) * mult / 2^32) with mult = floor(nh * 2^32 / range), nh = 7/8 of the
+// S/8 buckets: monotone in col, < nh, a multiply per product instead of a 64-bit division.
+__device__ __forceinline__ uint64_t bkt_mult(uint32_t range, uint32_t S) {
+  const uint64_t nb = S >> 3, nh = nb - (nb >> 3);
+  return range ? (nh << 32) / range : 0;
 }
-__device__ __forceinline__ uint32_t mono_slot(uint32_t col, uint32_t lo, uint64_t mult) {
+__device__ __forceinline__ uint32_t bkt_home(uint32_t col, uint32_t lo, uint64_t mult) {
   return (uint32_t)(((uint64_t)(col - lo) * mult) >> 32);
+}
+
+// Insert into the bucketed ordered map (keys 16-byte aligned, NB = S/8 buckets): two 16-byte
+// shared loads examine a bucket; a wrap-around past the last bucket (breaks the run order) is
+// reported.  Returns the key's slot.
+__device__ __forceinline__ uint32_t probe_insert_bkt(uint32_t* keys, uint32_t NB, uint32_t b, uint32_t key, int* wrapped) {
+  while (true) {
+    uint32_t k[8];
+    const uint32_t a = (uint32_t)__cvta_generic_to_shared(keys + 8 * b);
+    asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(k[0]), "=r"(k[1]), "=r"(k[2]), "=r"(k[3]) : "r"(a));
+    asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(k[4]), "=r"(k[5]), "=r"(k[6]), "=r"(k[7]) : "r"(a + 16));
+    uint32_t hit = 0, emp = 0;
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+      hit |= (uint32_t)(k[i] == key) << i;
+      emp |= (uint32_t)(k[i] == kEmptyKey) << i;
+    }
+    if (hit) return 8 * b + __ffs(hit) - 1;
+    if (emp) {
+      const uint32_t s = 8 * b + __ffs(emp) - 1;
+      const uint32_t old = atomicCAS(&keys[s], kEmptyKey, key);
+      if (old == kEmptyKey || old == key) return s;
+      continue;   // the slot was taken by another key: re-read the bucket
+    }
+    if (++b == NB) { b = 0; *wrapped = 1; }
+  }
 }
 
 // linear probing that reports a wrap-around (which breaks the cluster order)
@@ -130,6 +159,23 @@ __device__ __forceinline__ int warp_write_ordered(const uint32_t* rk, const V* r
     const uint32_t k = s < S ? rk[s] : kEmptyKey;        // slots past w1 only bound runs
     const uint32_t occ = __ballot_sync(0xffffffffu, k != kEmptyKey);
     const uint32_t mine = occ & (w1 - c0 >= 32 ? 0xffffffffu : ((1u << (w1 - c0)) - 1u));
+    // fast path (warp-uniform): no full bucket in the window and no run entering it, so every
+    // run is its bucket: rank among the bucket's 8 keys by shuffles, no divergent walk
+    const uint32_t fullb = occ & (occ >> 1) & (occ >> 2) & (occ >> 3) & (occ >> 4) & (occ >> 5) & (occ >> 6) & (occ >> 7) &
+                           0x01010101u;
+    if (!fullb && carry == 0) {
+      int rank = 0;
+#pragma unroll
+      for (int d = 1; d < 8; ++d) rank += __shfl_sync(0xffffffffu, k, (lane & ~7) | ((lane + d) & 7)) < k;
+      if ((mine >> lane) & 1u) {
+        const int64_t o = ob + before + written + __popc(occ & ((1u << (lane & ~7)) - 1u)) + rank;
+        C_col[o] = (int32_t)k;
+        C_val[o] = rv[s];
+      }
+      written += __popc(mine);
+      carry = __clz(~occ);
+      continue;
+    }
     if ((mine >> lane) & 1u) {
       const uint32_t zb = ~occ & lt;
       const uint32_t rs = zb ? c0 + 32 - __clz(zb) : c0 - carry;
@@ -622,7 +668,8 @@ __device__ __noinline__ void block_sorted_write(uint32_t* keys, V* vals, uint32_
 // products, hash insert (symbolic: count new keys; numeric: equal keys of a warp step add in
 // rounds — the region is private, so no atomics on values), then the sorted write-out
 // (ordered map for rows > kSmallSeg entries, else rank counting).  Returns the symbolic count.
-template <int PASS, typename V>
+// MODE (numeric): 0 any row, 1 rows of <= kSmallSeg entries only, 2 larger rows only.
+template <int PASS, typename V, int MODE = 0>
 __device__ __forceinline__ int warp_row(const SpgemmArgs<V>& p, uint32_t* rk, V* rv, uint32_t S, int64_t a0, int alen,
                                         int32_t cmin, int32_t cmax, int32_t cnt, int64_t cbase,
                                         const PreBatch<V>* pre = nullptr) {
@@ -633,10 +680,10 @@ __device__ __forceinline__ int warp_row(const SpgemmArgs<V>& p, uint32_t* rk, V*
   }
   __syncwarp();
   const uint32_t mlo = (uint32_t)cmin;
-  const uint64_t mmult = mono_mult((uint32_t)(cmax - cmin + 1), S);
+  const uint64_t mmult = bkt_mult((uint32_t)(cmax - cmin + 1), S);
   // long rows use the order-preserving map (sorted write-out without a sort network);
   // short rows keep the scrambled hash (robust to clustered columns) and rank counting
-  const bool ordered = PASS == 1 && cnt > kSmallSeg;
+  const bool ordered = PASS == 1 && (MODE == 2 || (MODE == 0 && cnt > kSmallSeg));
   int newc = 0, wrapped = 0;
   expand_row<PASS, V>(
       p, a0, alen, 0, 1, [&](uint32_t col, V v, bool act) {
@@ -647,7 +694,8 @@ __device__ __forceinline__ int warp_row(const SpgemmArgs<V>& p, uint32_t* rk, V*
       const uint32_t lt = (1u << lane_id()) - 1u;
       uint32_t s = 0;
       if (act && !(peers & lt)) {
-        s = probe_insert_mono(rk, S, ordered ? mono_slot(col, mlo, mmult) : hash_slot(col, S), col, &wrapped);
+        s = ordered ? probe_insert_bkt(rk, S >> 3, bkt_home(col, mlo, mmult), col, &wrapped)
+                    : probe_insert_mono(rk, S, hash_slot(col, S), col, &wrapped);
       }
       s = __shfl_sync(0xffffffffu, s, __ffs(peers) - 1);   // the key's slot, from its first lane
       const int rank = __popc(peers & lt);
@@ -659,7 +707,7 @@ __device__ __forceinline__ int warp_row(const SpgemmArgs<V>& p, uint32_t* rk, V*
     }
   });
   if (PASS == 0) return warp_sum(newc);
-  if (ordered && !__any_sync(0xffffffffu, wrapped)) {
+  if (MODE != 1 && ordered && !__any_sync(0xffffffffu, wrapped)) {
     // ordered map: every entry goes to (occupied slots before its run) + (rank in the run)
     warp_write_ordered<V>(rk, rv, S, 0u, S, cbase, 0, p.C_col, p.C_val);
   } else {
@@ -837,7 +885,7 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
         uint32_t* rk = keys + rb;
         V* rv = vals + rb;
         const uint32_t mlo = (uint32_t)bm.rlo[r];
-        const uint64_t mmult = mono_mult((uint32_t)(bm.rhi[r] - bm.rlo[r] + 1), S);
+        const uint64_t mmult = bkt_mult((uint32_t)(bm.rhi[r] - bm.rlo[r] + 1), S);
         const bool ordered = bm.ordered;
         int newc = 0, wrapped = 0;
         expand_row<PASS, V, PASS == 0, true>(p, bm.astart[r], (int)(bm.aoff[r + 1] - bm.aoff[r]), warp_id(), NW,
@@ -847,8 +895,8 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
                               } else {
                                 uint32_t s = 0;
                                 if (act)
-                                  s = probe_insert_mono(rk, S, ordered ? mono_slot(col, mlo, mmult) : hash_slot(col, S),
-                                                        col, &wrapped);
+                                  s = ordered ? probe_insert_bkt(rk, S >> 3, bkt_home(col, mlo, mmult), col, &wrapped)
+                                              : probe_insert_mono(rk, S, hash_slot(col, S), col, &wrapped);
                                 bool leader;
                                 const V sum = warp_key_sum(col, v, leader);
                                 if (act && leader) atomicAdd(&rv[s], sum);
@@ -984,7 +1032,7 @@ __device__ __noinline__ void dense_row(const SpgemmArgs<V>& p, BlockMeta& bm, in
 // write-out scan only the slots a row can use.  Rows of the bin (p.rows) or, without global
 // load balancing, every row of A (p.rows == nullptr).
 // -----------------------------------------------------------------------------------
-template <int PASS, typename V>
+template <int PASS, typename V, int MODE>
 __global__ void __launch_bounds__(kWarpRowThreads, kWarpRowCtasPerSM)
     k_warp_rows(SpgemmArgs<V> p, unsigned long long* __restrict__ counter) {
   extern __shared__ __align__(16) unsigned char smem[];
@@ -1079,7 +1127,7 @@ __global__ void __launch_bounds__(kWarpRowThreads, kWarpRowCtasPerSM)
     row = rown;
     mv = mvn;
     fetch((int64_t)enn, rown, mvn);
-    const int c = warp_row<PASS, V>(p, rk, rv, S, a0, alen, cmn, cmx, (int32_t)(m3 - m2), m2, &bcur);
+    const int c = warp_row<PASS, V, MODE>(p, rk, rv, S, a0, alen, cmn, cmx, (int32_t)(m3 - m2), m2, &bcur);
     if (PASS == 0 && lane == 0) p.cnt[cur] = c;
     e = en;
     en = enn;
