@@ -253,13 +253,14 @@ __global__ void __launch_bounds__(kCfgThreads[kSegCfg], 1024 / kCfgThreads[kSegC
 //      and the row's C.val range is zeroed;
 //   3. values: every product's position is prefix[word] + popc(lower bits of its word), and
 //      a·b is added there with a global atomic (the row's C range stays in L2).
-// No column segments, no binary searches in B rows, no hash probing and no sort.  Both passes
-// rotate product chunks over all 32 warps (expand_row ALL): a hub row of B referenced by the
-// row is streamed by every warp, not by the one warp whose batch holds it.  Columns are
+// No column segments, no binary searches in B rows, no hash probing and no sort.  Hub rows of
+// B (>= kLongB entries) referenced by the row are streamed by all 32 warps from a shared list,
+// the other batches go round-robin over the warps, so no warp is left with a hub row alone.  Columns are
 // relative to lo = colmin & ~31; smem: bits (4 B/word) + per-word prefix within its 32-word
 // group (uint16) + per-group prefix (int32).
 // ------------------------------------------------------------------------------------
 constexpr int kBitmapThreads = 1024;
+constexpr int kListAvgLen = 256;   // products / nnz(A_i) below this: shared hub-row list, else ALL mode
 // 196 B of shared memory per 32-word group (128 bits + 4 prefix + 64 word prefixes)
 constexpr int64_t kBitmapMaxCols = (int64_t)(kCfgMapBytes[kNumCfg - 1] / 196) * 1024;
 
@@ -268,6 +269,7 @@ __global__ void __launch_bounds__(kBitmapThreads, 1) k_long_bitmap(SpgemmArgs<V>
   constexpr int T = kBitmapThreads, NW = T / 32;
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ int64_t part[NW + 1];
+  __shared__ LongList<V> longs;
   const int32_t row = a.cand[blockIdx.x];
   const int64_t ob = a.C_rp[row], cnt = a.C_rp[row + 1] - ob;
   if (cnt <= a.limit || !bitmap_row(a, row)) return;
@@ -281,14 +283,27 @@ __global__ void __launch_bounds__(kBitmapThreads, 1) k_long_bitmap(SpgemmArgs<V>
   const int64_t a0 = p.A_rp[row];
   const int alen = (int)(p.A_rp[row + 1] - a0);
   for (int i = tid; i < G * 32; i += T) bits[i] = 0u;
-  __syncthreads();
+  // Rows whose referenced B rows are long on average (C3: ~800) rotate every chunk over all
+  // warps, each warp reading every batch (ALL mode; the redundant batch loads are cheap next to
+  // the products).  Rows of A with many short references (C4: 200k NZ, ~20 products each) would
+  // pay 32x their A traffic that way: there hub rows of B (>= kLongB entries) go to a shared
+  // list streamed by all warps and the other batches go round-robin over the warps.
+  bool listed = false;
+  if (p.prods[row] < (int64_t)kListAvgLen * alen) listed = collect_long_rows<1, V>(p, a0, alen, longs);
+  else __syncthreads();
   // 1. structure
-  expand_row<0, V, true, true>(p, a0, alen, wp, NW, [&](uint32_t col, V, bool act) {
+  auto set_bit = [&](uint32_t col, V, bool act) {
     if (act) {
       const uint32_t c = col - lo;
       atomicOr(&bits[c >> 5], 1u << (c & 31));
     }
-  });
+  };
+  if (listed) {
+    expand_long_list<0, V>(p, longs, wp, NW, set_bit);
+    expand_row<0, V, true, false>(p, a0, alen, wp, NW, set_bit, FullRange(), nullptr, kLongB);
+  } else {
+    expand_row<0, V, true, true>(p, a0, alen, wp, NW, set_bit);
+  }
   __syncthreads();
   // 2. prefixes: warp w owns groups [w*GW, (w+1)*GW); lane i holds word i of a group
   const int GW = (G + NW - 1) / NW;
@@ -335,13 +350,19 @@ __global__ void __launch_bounds__(kBitmapThreads, 1) k_long_bitmap(SpgemmArgs<V>
   __syncthreads();
   // 3. values
   V* cv = p.C_val + ob;
-  expand_row<1, V, true, true>(p, a0, alen, wp, NW, [&](uint32_t col, V v, bool act) {
+  auto add_val = [&](uint32_t col, V v, bool act) {
     if (act) {
       const uint32_t c = col - lo, w = c >> 5;
       const int r = gpre[w >> 5] + (int)wpre[w] + __popc(bits[w] & ((1u << (c & 31)) - 1u));
       atomicAdd(cv + r, v);
     }
-  });
+  };
+  if (listed) {
+    expand_long_list<1, V>(p, longs, wp, NW, add_val);
+    expand_row<1, V, true, false>(p, a0, alen, wp, NW, add_val, FullRange(), nullptr, kLongB);
+  } else {
+    expand_row<1, V, true, true>(p, a0, alen, wp, NW, add_val);
+  }
 }
 
 }  // namespace speck

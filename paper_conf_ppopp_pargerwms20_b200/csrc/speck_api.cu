@@ -355,10 +355,13 @@ SegPlanArgs seg_plan_args(speck_handle_t h, const int64_t* C_rp) {
   s.dense_window = num_dense_window<V>(kSegCfg);
   s.map_slots = num_map_cap<V>(kSegCfg);
   s.seg_limit = num_map_fill<V>(kSegCfg);
-  // few candidates: split every long row so its work spreads over the SMs
-  s.prefer_parallel = h->n_cand < 4 * (int64_t)h->num_sms ? 1 : 0;
+  // few candidates: split every long row so its work spreads over the SMs — unless rows of A
+  // are very long: every column segment binary-searches each referenced B row, so a segment
+  // costs O(nnz(A_i)) before its first product (C4: 200k-NZ rows, 32 segments each; the bitmap
+  // CTA per row took the numeric step 32.6 -> 16.5 ms)
+  s.prefer_parallel = (h->n_cand < 4 * (int64_t)h->num_sms && h->max_nnza < kSegMaxNnzA) ? 1 : 0;
   // many long rows: one bitmap CTA per row whose column range fits (no column segments)
-  s.bitmap_cols = (h->opt_long_bitmap && !s.prefer_parallel) ? kBitmapMaxCols : 0;
+  s.bitmap_cols = (h->opt_long_bitmap == 2 || (h->opt_long_bitmap && !s.prefer_parallel)) ? kBitmapMaxCols : 0;
   return s;
 }
 

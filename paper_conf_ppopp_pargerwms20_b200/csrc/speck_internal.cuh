@@ -58,6 +58,8 @@ constexpr int kMaxChunks = 1024;
 // Long-row jobs run in configuration 3 (512 threads, 2 CTAs per SM), so one CTA's barriers
 // overlap with the other's work; segments hold up to that map's fill.
 constexpr int kSegCfg = kNumCfg - 2;
+// rows of A longer than this make column segments expensive (see seg_plan_args)
+constexpr int64_t kSegMaxNnzA = 16384;
 struct Seg {
   int32_t row;
   int32_t col_lo;   // first column of the segment

@@ -360,7 +360,7 @@ struct PreBatch {
 // or write the same value from every warp.
 template <int PASS, typename V, bool STREAM = (PASS == 0), bool ALL = false, typename Ins, typename Rng = FullRange>
 __device__ __forceinline__ void expand_row(const SpgemmArgs<V>& p, int64_t a0, int alen, int wi, int nw, Ins&& ins,
-                                           Rng rng = Rng(), const PreBatch<V>* pre = nullptr) {
+                                           Rng rng = Rng(), const PreBatch<V>* pre = nullptr, int skip_len = 0) {
   const int lane = lane_id();
   const int nb = (alen + 31) >> 5;
   constexpr int CH = 32 * kPPL;
@@ -393,6 +393,7 @@ __device__ __forceinline__ void expand_row(const SpgemmArgs<V>& p, int64_t a0, i
       rng(f, p.B_rp[kc], p.B_rp[kc + 1], s, e);
       bst = s;
       blen = (int)(e - s);
+      if (skip_len > 0 && blen >= skip_len) blen = 0;   // taken from the caller's shared list
     }
     // STREAM (symbolic, long-row bitmap kernel): long referenced B rows (>= kStreamLen
     // products) are streamed by the warp directly — contiguous, coalesced loads, no owner
@@ -465,6 +466,70 @@ __device__ __forceinline__ void expand_row(const SpgemmArgs<V>& p, int64_t a0, i
         if (p0 + 32 * i >= Pb) continue;   // uniform skip of empty sub-chunks
         const V ao = PASS == 1 ? __shfl_sync(0xffffffffu, a, oa[i]) : V(0);
         ins(ca[i], ao * va[i], p0 + lane + 32 * i < Pb);
+      }
+    }
+  }
+}
+
+// Referenced B rows of at least kLongB entries collected into a shared list (collect_long_rows)
+// and streamed by all nw warps, product chunks rotated over the warps (no redundant batch
+// loads, unlike expand_row's ALL mode, which re-reads every batch in every warp: for C4's
+// 200k-NZ rows of A that was 32x the A traffic).
+constexpr int kLongB = 1024;
+constexpr int kLongListCap = 128;
+template <typename V>
+struct LongList {
+  int64_t bst[kLongListCap];
+  int32_t len[kLongListCap];
+  V a[kLongListCap];
+  int n;
+};
+// All threads of the block; barriers inside.  Returns true if every long row fit the list.
+template <int PASS, typename V>
+__device__ bool collect_long_rows(const SpgemmArgs<V>& p, int64_t a0, int alen, LongList<V>& L) {
+  if (threadIdx.x == 0) L.n = 0;
+  __syncthreads();
+  for (int f = threadIdx.x; f < alen; f += blockDim.x) {
+    const int32_t kc = p.A_col[a0 + f];
+    const int64_t b0 = p.B_rp[kc];
+    const int len = (int)(p.B_rp[kc + 1] - b0);
+    if (len >= kLongB) {
+      const int i = atomicAdd(&L.n, 1);
+      if (i < kLongListCap) {
+        L.bst[i] = b0;
+        L.len[i] = len;
+        L.a[i] = PASS == 1 ? ldv(p.A_val + a0 + f) : V(0);
+      }
+    }
+  }
+  __syncthreads();
+  return L.n <= kLongListCap;
+}
+template <int PASS, typename V, typename Ins>
+__device__ __forceinline__ void expand_long_list(const SpgemmArgs<V>& p, const LongList<V>& L, int wi, int nw, Ins&& ins) {
+  constexpr int CH = 32 * kPPL;
+  const int lane = lane_id();
+  int rot = 0;
+  for (int r = 0; r < L.n; ++r) {
+    const int len = L.len[r];
+    const int64_t s0 = L.bst[r];
+    const V ao = L.a[r];
+    const int nsub = (len + CH - 1) / CH;
+    const int j0 = (wi - rot + nw) % nw;
+    rot = (rot + nsub) % nw;
+    for (int q0 = j0 * CH; q0 < len; q0 += nw * CH) {
+      uint32_t c[kPPL];
+      V bv[kPPL];
+#pragma unroll
+      for (int i = 0; i < kPPL; ++i) {
+        const int q = q0 + 32 * i + lane;
+        c[i] = q < len ? (uint32_t)p.B_col[s0 + q] : (0x80000000u | (uint32_t)lane);
+        bv[i] = (PASS == 1 && q < len) ? ldv(p.B_val + s0 + q) : V(0);
+      }
+#pragma unroll
+      for (int i = 0; i < kPPL; ++i) {
+        if (q0 + 32 * i >= len) continue;   // warp-uniform
+        ins(c[i], ao * bv[i], q0 + 32 * i + lane < len);
       }
     }
   }
