@@ -88,7 +88,9 @@ typedef enum {
   SPECK_OPT_CONCURRENT_STREAMS = 8, /* number of internal streams for concurrent bins, 1..8 [4] */
   SPECK_OPT_SEGMENTS = 9,           /* 1: split rows beyond the largest map into column segments; 0: windowed dense [1] */
   SPECK_OPT_WARP_ROWS = 10,         /* 1: smallest bin = one warp per row (k_warp_rows); 0: merged blocks (Alg. 2) [1] */
-  SPECK_OPT_LONG_BITMAP = 11        /* 1: many long rows -> one bitmap+rank CTA per row when the column range fits [1] */
+  SPECK_OPT_LONG_BITMAP = 11,       /* 1: many long rows -> one bitmap+rank CTA per row when the column range fits; 2: always [1] */
+  SPECK_OPT_BITMAP_REUSE = 12       /* 1: the symbolic step keeps the dense bitmaps of numeric long rows (workspace
+                                       <= 1/4 of free memory) so the numeric step does not rebuild them [1] */
 } speck_option_t;
 
 /* Statistics of the last analyze/spgemm pair (speck_get_stats). */

@@ -64,6 +64,8 @@ struct SegPlanArgs {
   int64_t map_slots;       // slots of the largest numeric hash map
   int prefer_parallel;     // few long rows: always split (parallelism across SMs)
   int64_t bitmap_cols;     // >0: rows whose column range fits are done by k_long_bitmap (no segments)
+  const uint32_t* bm_pool; // bitmaps kept by the symbolic step (SpgemmArgs::bm_pool), or null
+  const int64_t* bm_off;   // per candidate: word offset in bm_pool, -1 = rebuild
 };
 
 // Long rows whose column range fits the shared-memory bitmap of k_long_bitmap.
@@ -260,7 +262,6 @@ __global__ void __launch_bounds__(kCfgThreads[kSegCfg], 1024 / kCfgThreads[kSegC
 // group (uint16) + per-group prefix (int32).
 // ------------------------------------------------------------------------------------
 constexpr int kBitmapThreads = 1024;
-constexpr int kListAvgLen = 256;   // products / nnz(A_i) below this: shared hub-row list, else ALL mode
 // 196 B of shared memory per 32-word group (128 bits + 4 prefix + 64 word prefixes)
 constexpr int64_t kBitmapMaxCols = (int64_t)(kCfgMapBytes[kNumCfg - 1] / 196) * 1024;
 
@@ -282,14 +283,21 @@ __global__ void __launch_bounds__(kBitmapThreads, 1) k_long_bitmap(SpgemmArgs<V>
   uint16_t* wpre = reinterpret_cast<uint16_t*>(smem + (size_t)G * 128 + (size_t)G * 4);
   const int64_t a0 = p.A_rp[row];
   const int alen = (int)(p.A_rp[row + 1] - a0);
-  for (int i = tid; i < G * 32; i += T) bits[i] = 0u;
+  const long long bmo = a.bm_pool ? a.bm_off[blockIdx.x] : -1ll;
+  if (bmo >= 0) {
+    // the symbolic step kept this row's bitmap: load it instead of rebuilding it (pass 1)
+    const uint32_t* src = a.bm_pool + bmo;
+    for (int i = tid; i < G * 32; i += T) bits[i] = i < W ? __ldcs(src + i) : 0u;
+  } else {
+    for (int i = tid; i < G * 32; i += T) bits[i] = 0u;
+  }
   // Rows whose referenced B rows are long on average (C3: ~800) rotate every chunk over all
   // warps, each warp reading every batch (ALL mode; the redundant batch loads are cheap next to
   // the products).  Rows of A with many short references (C4: 200k NZ, ~20 products each) would
   // pay 32x their A traffic that way: there hub rows of B (>= kLongB entries) go to a shared
   // list streamed by all warps and the other batches go round-robin over the warps.
   bool listed = false;
-  if (p.prods[row] < (int64_t)kListAvgLen * alen) listed = collect_long_rows<1, V>(p, a0, alen, longs);
+  if (p.prods[row] < (int64_t)kAllAvgLen * alen) listed = collect_long_rows<1, V>(p, a0, alen, longs);
   else __syncthreads();
   // 1. structure
   auto set_bit = [&](uint32_t col, V, bool act) {
@@ -298,7 +306,8 @@ __global__ void __launch_bounds__(kBitmapThreads, 1) k_long_bitmap(SpgemmArgs<V>
       atomicOr(&bits[c >> 5], 1u << (c & 31));
     }
   };
-  if (listed) {
+  if (bmo >= 0) {
+  } else if (listed) {
     expand_long_list<0, V>(p, longs, wp, NW, set_bit);
     expand_row<0, V, true, false>(p, a0, alen, wp, NW, set_bit, FullRange(), nullptr, kLongB);
   } else {

@@ -63,6 +63,10 @@ struct speck_handle_s {
   int64_t opt_segments = 1;
   int64_t opt_warp_rows = 1;
   int64_t opt_long_bitmap = 1;
+  int64_t opt_bitmap_reuse = 1;
+  bool bm_enabled = false;
+  unsigned long long bm_pool_words = 0;
+  Buf bm_pool, bm_off;
   bool seg_enabled = false;
   int seg_shift = 15, nchunks = 0;
   int64_t long_thr = INT64_MAX, n_cand = 0, n_segs = 0, cand_start = 0;
@@ -100,12 +104,12 @@ speck_status_t fail(speck_handle_t h, speck_status_t s, const char* fmt, ...) {
                   __FILE__, __LINE__);                                                                \
   } while (0)
 
-speck_status_t ensure(speck_handle_t h, Buf& b, size_t bytes, cudaStream_t s) {
+speck_status_t ensure(speck_handle_t h, Buf& b, size_t bytes, cudaStream_t s, bool exact = false) {
   if (bytes <= b.cap) return SPECK_OK;
   if (b.p) CK(cudaFreeAsync(b.p, s));
   b.p = nullptr;
   b.cap = 0;
-  size_t want = std::max<size_t>(bytes + bytes / 4, 4096);
+  size_t want = std::max<size_t>(exact ? bytes : bytes + bytes / 4, 4096);
   cudaError_t e = cudaMallocAsync(&b.p, want, s);
   if (e != cudaSuccess) {
     (void)cudaGetLastError();
@@ -119,7 +123,8 @@ speck_status_t ensure(speck_handle_t h, Buf& b, size_t bytes, cudaStream_t s) {
 int64_t ws_bytes(speck_handle_t h) {
   return (int64_t)(h->prods.cap + h->maxlen.cap + h->colmin.cap + h->colmax.cap + h->cnt.cap + h->hist.cap +
                    h->hist_off.cap + h->bins.cap + h->stats.cap + h->scan_status.cap + h->resume.cap + h->small.cap +
-                   h->ana_long.cap + h->chunk_cnt.cap + h->cand.cap + h->nseg.cap + h->seg_off.cap + h->segs.cap);
+                   h->ana_long.cap + h->chunk_cnt.cap + h->cand.cap + h->nseg.cap + h->seg_off.cap + h->segs.cap +
+                   h->bm_pool.cap + h->bm_off.cap);
 }
 
 speck_status_t check_csr(speck_handle_t h, const speck_csr_t* M, const char* name, bool need_values) {
@@ -362,6 +367,8 @@ SegPlanArgs seg_plan_args(speck_handle_t h, const int64_t* C_rp) {
   s.prefer_parallel = (h->n_cand < 4 * (int64_t)h->num_sms && h->max_nnza < kSegMaxNnzA) ? 1 : 0;
   // many long rows: one bitmap CTA per row whose column range fits (no column segments)
   s.bitmap_cols = (h->opt_long_bitmap == 2 || (h->opt_long_bitmap && !s.prefer_parallel)) ? kBitmapMaxCols : 0;
+  s.bm_pool = (h->bm_enabled && s.bitmap_cols > 0) ? static_cast<const uint32_t*>(h->bm_pool.p) : nullptr;
+  s.bm_off = static_cast<const int64_t*>(h->bm_off.p);
   return s;
 }
 
@@ -452,6 +459,12 @@ speck_status_t run_pass(speck_handle_t h, int pass, int lb, const int64_t* cat_s
       b.nchunks = h->nchunks;
       b.chunk_shift = h->seg_shift;
       b.long_thr = h->long_thr;
+      if (h->bm_enabled) {
+        b.bm_pool = static_cast<uint32_t*>(h->bm_pool.p);
+        b.bm_pool_words = h->bm_pool_words;
+        b.bm_ctr = reinterpret_cast<unsigned long long*>(static_cast<char*>(h->small.p) + 2048);
+        b.bm_off = static_cast<int64_t*>(h->bm_off.p);
+      }
     }
     st = launch_spgemm<V>(h, c, pass, b, h->streams[si]);
     if (st) return st;
@@ -604,6 +617,31 @@ speck_status_t analyze_impl(speck_handle_t h, const speck_csr_t* A, const speck_
     }
   } else {
     h->n_cand = 0;
+  }
+  // bitmap reuse: will the numeric long rows go to k_long_bitmap (seg_plan_args), and does every
+  // row's column range fit its bitmap?  Then the symbolic dense rows keep their bitmaps.
+  h->bm_enabled = false;
+  if (h->seg_enabled && h->n_cand > 0 && h->opt_bitmap_reuse && h->opt_long_bitmap && B->cols <= kBitmapMaxCols &&
+      (h->opt_long_bitmap == 2 || !(h->n_cand < 4 * (int64_t)h->num_sms && h->max_nnza < kSegMaxNnzA))) {
+    const size_t per_row = ((size_t)(B->cols + 31) / 32 + 4) * 4;
+    size_t want = ((size_t)h->n_cand * per_row + 15) & ~(size_t)15;
+    if (want > h->bm_pool.cap) {
+      // growing: cap the pool at a quarter of the free memory (C is allocated after analyze);
+      // the query is slow, so it only happens when the pool grows
+      size_t free_b = 0, tot_b = 0;
+      CK(cudaMemGetInfo(&free_b, &tot_b));
+      want = std::min<size_t>(want, (free_b + h->bm_pool.cap) / 4) & ~(size_t)15;
+      if (want < h->bm_pool.cap) want = h->bm_pool.cap;
+    }
+    if (want >= ((size_t)1 << 20) && ensure(h, h->bm_pool, want, s, true) == SPECK_OK &&
+        ensure(h, h->bm_off, (size_t)h->n_cand * 8, s) == SPECK_OK) {
+      CK(cudaMemsetAsync(h->bm_off.p, 0xFF, (size_t)h->n_cand * 8, s));
+      CK(cudaMemsetAsync(static_cast<char*>(h->small.p) + 2048, 0, 8, s));
+      h->bm_pool_words = h->bm_pool.cap / 4;
+      h->bm_enabled = true;
+    } else {
+      (void)cudaGetLastError();
+    }
   }
   SpgemmArgs<V> a = base_args<V>(h, A, B);
   if (lb_sym) {
@@ -815,7 +853,7 @@ speck_status_t speck_destroy(speck_handle_t h) {
   cudaDeviceSynchronize();
   Buf* bufs[] = {&h->prods, &h->maxlen, &h->colmin, &h->colmax, &h->cnt, &h->hist, &h->hist_off, &h->bins, &h->stats,
                  &h->scan_status, &h->resume, &h->small, &h->ana_long, &h->chunk_cnt, &h->cand, &h->nseg,
-                 &h->seg_off, &h->segs};
+                 &h->seg_off, &h->segs, &h->bm_pool, &h->bm_off};
   for (Buf* b : bufs)
     if (b->p) cudaFree(b->p);
   if (h->h_pinned) cudaFreeHost(h->h_pinned);
@@ -855,6 +893,7 @@ speck_status_t speck_set_option(speck_handle_t h, int option, int64_t v) {
     case SPECK_OPT_SEGMENTS: h->opt_segments = v; break;
     case SPECK_OPT_WARP_ROWS: h->opt_warp_rows = v; break;
     case SPECK_OPT_LONG_BITMAP: h->opt_long_bitmap = v; break;
+    case SPECK_OPT_BITMAP_REUSE: h->opt_bitmap_reuse = v; break;
     default: return fail(h, SPECK_ERR_INVALID_ARGUMENT, "unknown option %d", option);
   }
   return SPECK_OK;

@@ -312,6 +312,12 @@ struct SpgemmArgs {
   int nchunks;
   int chunk_shift;           // chunk = col >> chunk_shift
   int64_t long_thr;          // rows with prods > long_thr record chunk counts
+  // symbolic, largest configuration: the dense bitmap of a row that will be a numeric long row
+  // is kept in a pool for k_long_bitmap (bm_off[entry] = word offset, -1 if not kept)
+  uint32_t* bm_pool;
+  unsigned long long bm_pool_words;
+  unsigned long long* bm_ctr;
+  int64_t* bm_off;
 };
 
 }  // namespace speck

@@ -28,6 +28,7 @@ namespace speck {
 
 constexpr int kSmallSeg = kTinyCnt;   // rows with <= this many C entries are ranked, not sorted
 constexpr int kPPL = 4;         // products per lane per chunk in the warp-per-row path
+constexpr int kAllAvgLen = 256;  // expand_row ALL mode for rows whose references average >= this many products
 constexpr int kStreamLen = 64;  // referenced B rows at least this long are streamed, not balanced
 
 struct BlockMeta {
@@ -1055,7 +1056,10 @@ __device__ __noinline__ void dense_row(const SpgemmArgs<V>& p, BlockMeta& bm, in
         __syncthreads();
         // expand-balanced accumulation of the products falling into this window
         auto ins = [&](uint32_t col, V v, bool act) { dense_insert<PASS, V>(bits, dvals, (uint32_t)wlo, col, v, act); };
-        if (nwin == 1) expand_row<PASS, V, PASS == 0, true>(p, astart, (int)nnzA, warp_id(), NW, ins);
+        // ALL mode (every warp reads every batch) only where references are long on average:
+        // C4's 200k-NZ rows of A with ~20 products per reference paid 32x their A traffic
+        if (nwin == 1 && bm.prods >= kAllAvgLen * nnzA) expand_row<PASS, V, PASS == 0, true>(p, astart, (int)nnzA, warp_id(), NW, ins);
+        else if (nwin == 1) expand_row<PASS, V>(p, astart, (int)nnzA, warp_id(), NW, ins);
         else expand_row<PASS, V>(p, astart, (int)nnzA, warp_id(), NW, ins, WindowRange{res, res_next, p.B_col, (uint32_t)whi});
         __syncthreads();
         { int32_t* t_ = res; res = res_next; res_next = t_; }
@@ -1080,6 +1084,23 @@ __device__ __noinline__ void dense_row(const SpgemmArgs<V>& p, BlockMeta& bm, in
         __syncthreads();
       }
       if (PASS == 0 && tid == 0) p.cnt[row] = total;
+      if (CFG == kNumCfg - 1 && PASS == 0 && chunks && p.bm_pool && nwin == 1 && total > p.long_thr) {
+        // keep the bitmap (words relative to colmin & ~31, as k_long_bitmap lays it out)
+        const int nwords = (int)((hi - lo + 1 + 31) / 32);
+        __shared__ long long s_bmo;
+        if (tid == 0) {
+          const unsigned long long need = ((unsigned long long)nwords + 3ull) & ~3ull;
+          const unsigned long long o = atomicAdd(p.bm_ctr, need);
+          s_bmo = o + need <= p.bm_pool_words ? (long long)o : -1ll;
+          p.bm_off[blockIdx.x] = s_bmo;
+        }
+        __syncthreads();
+        const long long o = s_bmo;
+        if (o >= 0) {
+          uint32_t* dst = p.bm_pool + o;
+          for (int i = tid; i < nwords; i += T) dst[i] = bits[i];
+        }
+      }
       if (chunks) {
         int32_t* dst = p.chunk_cnt + (int64_t)blockIdx.x * p.nchunks;
         for (int i = tid; i < p.nchunks; i += T) dst[i] = chist[i];

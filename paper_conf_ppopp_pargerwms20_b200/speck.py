@@ -23,7 +23,7 @@ SPECK_F32, SPECK_F64 = 0, 1
 OPT = {
     "global_lb_symbolic": 0, "global_lb_numeric": 1, "force_accumulator": 2, "dense_window": 3,
     "stage_timing": 4, "validate": 5, "disable_direct": 6, "fixed_group_size": 7, "concurrent_streams": 8,
-    "segments": 9, "warp_rows": 10, "long_bitmap": 11,
+    "segments": 9, "warp_rows": 10, "long_bitmap": 11, "bitmap_reuse": 12,
 }
 STATUS = {
     0: "SPECK_OK", 1: "SPECK_ERR_INVALID_ARGUMENT", 2: "SPECK_ERR_DIMENSION_MISMATCH", 3: "SPECK_ERR_DTYPE_MISMATCH",

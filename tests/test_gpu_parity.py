@@ -236,6 +236,56 @@ def test_many_long_rows_bitmap(dev, long_bitmap, dt):
     assert_parity(A, B, C)
 
 
+@pytest.mark.parametrize("reuse", [1, 0])
+@pytest.mark.parametrize("dt", [torch.float32, torch.float64])
+def test_bitmap_reuse(dev, reuse, dt):
+    """Many long rows whose column ranges all fit the bitmap (B has 2^20 columns): the symbolic
+    step keeps each long row's dense bitmap and k_long_bitmap loads it instead of rebuilding it
+    (bitmap_reuse=1), or rebuilds it (0).  Both must match the oracle."""
+    import numpy as _np
+    rng = _np.random.default_rng(17)
+    nb, lb = 3000, 1000
+    cols = np.stack([np.sort(rng.choice(1 << 20, size=lb, replace=False)) for _ in range(nb)])
+    B = W.csr_from_coo(nb, 1 << 20, torch.arange(nb).repeat_interleave(lb), torch.tensor(cols.reshape(-1)), None,
+                       dtype=dt, seed=18)
+    ar = np.repeat(np.arange(700), 24)
+    ac = np.concatenate([np.sort(rng.choice(nb, 24, replace=False)) for _ in range(700)])
+    A = W.csr_from_coo(700, nb, torch.tensor(ar), torch.tensor(ac), None, dtype=dt, seed=19)
+    C, st = gpu_spgemm(A, B, bitmap_reuse=reuse)
+    assert st["rows_per_bin_numeric"][7] >= 600
+    assert_parity(A, B, C)
+    # handle reuse: a second analyze/spgemm pair on the same handle reuses the pool
+    h = sp.Handle(0, bitmap_reuse=reuse)
+    for _ in range(2):
+        C2 = h.spgemm(A.to("cuda"), B.to("cuda"))
+    torch.cuda.synchronize()
+    h.close()
+    assert torch.equal(C2.col.cpu(), C.col.cpu())
+
+
+@pytest.mark.parametrize("dt", [torch.float32, torch.float64])
+def test_very_long_rows_of_a(dev, dt):
+    """C4-like: a few rows of A with 20k NZ (over 2^16 columns of B, rows of 8 entries, plus a few
+    hub rows of 5000 entries) -> long rows of C handled by the bitmap CTA with the shared hub-row
+    list (segments would binary-search every referenced B row per segment)."""
+    import numpy as _np
+    rng = _np.random.default_rng(23)
+    nb = 40_000
+    lens = np.full(nb, 8)
+    lens[rng.choice(nb, 20, replace=False)] = 5000
+    rows = np.repeat(np.arange(nb), lens)
+    bc = np.concatenate([np.sort(rng.choice(1 << 16, size=int(l), replace=False)) for l in lens])
+    B = W.csr_from_coo(nb, 1 << 16, torch.tensor(rows), torch.tensor(bc), None, dtype=dt, seed=24)
+    na = 40
+    alen = np.where(np.arange(na) < 4, 20_000, 8)
+    ar = np.repeat(np.arange(na), alen)
+    ac = np.concatenate([np.sort(rng.choice(nb, size=int(l), replace=False)) for l in alen])
+    A = W.csr_from_coo(na, nb, torch.tensor(ar), torch.tensor(ac), None, dtype=dt, seed=25)
+    C, st = gpu_spgemm(A, B)
+    assert st["rows_per_bin_numeric"][7] >= 4
+    assert_parity(A, B, C)
+
+
 def test_fig5_dense_window_of_three(dev):
     """Fig. 5: one row, 6 columns, window 3, products at c0,c2,c4,c4,c5 -> c0=1 c2=1 c4=2 c5=1."""
     kv, _ = golden("fig5_dense.txt")
