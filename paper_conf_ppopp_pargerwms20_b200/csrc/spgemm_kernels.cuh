@@ -431,6 +431,7 @@ __device__ __forceinline__ void expand_row(const SpgemmArgs<V>& p, int64_t a0, i
     const int incl = warp_incl_scan(blen);
     const int excl = incl - blen;
     const int Pb = __shfl_sync(0xffffffffu, incl, 31);
+    const int64_t boff = bst - excl;   // product pp of owner o is B entry boff_o + pp
     // locate the products of chunk q0 and issue their loads (not consumed here)
     auto gather = [&](int q0, uint32_t (&c)[kPPL], V (&bv)[kPPL], int (&ow)[kPPL]) {
 #pragma unroll
@@ -447,7 +448,7 @@ __device__ __forceinline__ void expand_row(const SpgemmArgs<V>& p, int64_t a0, i
           if (probe <= pp) lo += step;
         }
         const int o = lo > 31 ? 31 : lo;
-        const int64_t idx = __shfl_sync(0xffffffffu, bst, o) + (pp - __shfl_sync(0xffffffffu, excl, o));
+        const int64_t idx = __shfl_sync(0xffffffffu, boff, o) + pp;
         ow[i] = o;
         if (pp < Pb) {
           c[i] = (uint32_t)p.B_col[idx];
@@ -1128,6 +1129,7 @@ __global__ void __launch_bounds__(kWarpRowThreads, kWarpRowCtasPerSM)
   V* rv = reinterpret_cast<V*>(region + (PASS == 0 ? 0u : wr_num_val_offset<V>()));
   const uint32_t cap = PASS == 0 ? wr_sym_cap() : wr_num_cap<V>();
   const int64_t n = p.n_entries;
+  constexpr bool kRange = PASS == 1 && MODE != 1;
   // row metadata, one field per lane: 0 A_rp[r], 1 A_rp[r+1], 2 prods[r] / C_rp[r], 3 C_rp[r+1],
   // 4 colmin[r], 5 colmax[r] (one round trip instead of six dependent loads)
   auto fetch = [&](int64_t e, int32_t& row, int64_t& mv) {
@@ -1139,8 +1141,8 @@ __global__ void __launch_bounds__(kWarpRowThreads, kWarpRowCtasPerSM)
       else if (lane == 1) mv = p.A_rp[row + 1];
       else if (lane == 2) mv = PASS == 0 ? p.prods[row] : p.C_rp[row];
       else if (lane == 3 && PASS == 1) mv = p.C_rp[row + 1];
-      else if (lane == 4) mv = p.colmin[row];
-      else if (lane == 5) mv = p.colmax[row];
+      else if (lane == 4 && kRange) mv = p.colmin[row];   // column range: ordered maps only
+      else if (lane == 5 && kRange) mv = p.colmax[row];
     }
   };
   // rows are claimed kWarpRowChunk at a time (one same-address atomic per chunk: per-row
