@@ -859,7 +859,7 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
       // (C5: the write-out scan of the full map was over half of the numeric instructions).
       if (l < nr) {
         if (nr == 1) {
-          const uint64_t want = (uint64_t)need * 2;
+          const uint64_t want = PASS == 0 ? (uint64_t)need * 2 : (uint64_t)need * 5 / 2;
           const uint64_t w32 = (want + 31) & ~(uint64_t)31;
           rsz = (uint32_t)(w32 < 64 ? 64 : (w32 > cap ? cap : w32));
         } else {
@@ -1202,7 +1202,7 @@ __global__ void __launch_bounds__(kWarpRowThreads, kWarpRowCtasPerSM)
     const int32_t cur = row;
     const int64_t need = PASS == 0 ? m2 : m3 - m2;       // products (symbolic) / exact nnz (numeric)
     // region: symbolic 1.5x products (66% fill), numeric 2x entries (50% fill), 32-slot multiples
-    const uint64_t want = (uint64_t)need * 2;
+    const uint64_t want = PASS == 0 ? (uint64_t)need * 2 : (uint64_t)need * 5 / 2;
     const uint64_t w32 = (want + 31) & ~(uint64_t)31;
     const uint32_t S = (uint32_t)(w32 < 64 ? 64 : (w32 > cap ? cap : w32));
     const PreBatch<V> bcur = bt;
