@@ -359,12 +359,13 @@ struct PreBatch {
 // hub row of B (ncu, C5: 22-50% of the stall samples of the single-row kernels were that
 // barrier with batches assigned round-robin).  Rng must then be pure (evaluated by every warp)
 // or write the same value from every warp.
-template <int PASS, typename V, bool STREAM = (PASS == 0), bool ALL = false, typename Ins, typename Rng = FullRange>
+template <int PASS, typename V, bool STREAM = (PASS == 0), bool ALL = false, int PPL = kPPL, typename Ins,
+          typename Rng = FullRange>
 __device__ __forceinline__ void expand_row(const SpgemmArgs<V>& p, int64_t a0, int alen, int wi, int nw, Ins&& ins,
                                            Rng rng = Rng(), const PreBatch<V>* pre = nullptr, int skip_len = 0) {
   const int lane = lane_id();
   const int nb = (alen + 31) >> 5;
-  constexpr int CH = 32 * kPPL;
+  constexpr int CH = 32 * PPL;
   // fewer batches than warps: G = nw/nb warps per batch, splitting its product chunks;
   // otherwise batches go round-robin and a warp takes all chunks of its batch
   const int G = ALL ? nw : (nb >= nw ? 1 : nw / nb);
@@ -411,16 +412,16 @@ __device__ __forceinline__ void expand_row(const SpgemmArgs<V>& p, int64_t a0, i
         const V ao = PASS == 1 ? __shfl_sync(0xffffffffu, a, o) : V(0);
         if (ALL) c_first = my_first((L + CH - 1) / CH);
         for (int q0 = c_first * CH; q0 < L; q0 += c_step * CH) {
-          uint32_t c[kPPL];
-          V bv[kPPL];
+          uint32_t c[PPL];
+          V bv[PPL];
 #pragma unroll
-          for (int i = 0; i < kPPL; ++i) {
+          for (int i = 0; i < PPL; ++i) {
             const int q = q0 + 32 * i + lane;
             c[i] = q < L ? (uint32_t)p.B_col[s0 + q] : (0x80000000u | (uint32_t)lane);
             bv[i] = (PASS == 1 && q < L) ? ldv(p.B_val + s0 + q) : V(0);
           }
 #pragma unroll
-          for (int i = 0; i < kPPL; ++i) {
+          for (int i = 0; i < PPL; ++i) {
             if (q0 + 32 * i >= L) continue;   // warp-uniform
             ins(c[i], ao * bv[i], q0 + 32 * i + lane < L);
           }
@@ -433,9 +434,9 @@ __device__ __forceinline__ void expand_row(const SpgemmArgs<V>& p, int64_t a0, i
     const int Pb = __shfl_sync(0xffffffffu, incl, 31);
     const int64_t boff = bst - excl;   // product pp of owner o is B entry boff_o + pp
     // locate the products of chunk q0 and issue their loads (not consumed here)
-    auto gather = [&](int q0, uint32_t (&c)[kPPL], V (&bv)[kPPL], int (&ow)[kPPL]) {
+    auto gather = [&](int q0, uint32_t (&c)[PPL], V (&bv)[PPL], int (&ow)[PPL]) {
 #pragma unroll
-      for (int i = 0; i < kPPL; ++i) {
+      for (int i = 0; i < PPL; ++i) {
         c[i] = 0x80000000u | (uint32_t)lane;   // inactive lanes keep a key that is never a real column
         bv[i] = V(0);
         ow[i] = 0;
@@ -456,15 +457,15 @@ __device__ __forceinline__ void expand_row(const SpgemmArgs<V>& p, int64_t a0, i
         }
       }
     };
-    // gather a chunk (kPPL independent loads per lane), then insert it
-    uint32_t ca[kPPL];
-    V va[kPPL];
-    int oa[kPPL];
+    // gather a chunk (PPL independent loads per lane), then insert it
+    uint32_t ca[PPL];
+    V va[PPL];
+    int oa[PPL];
     if (ALL) c_first = my_first((Pb + CH - 1) / CH);
     for (int p0 = c_first * CH; p0 < Pb; p0 += c_step * CH) {
       gather(p0, ca, va, oa);
 #pragma unroll
-      for (int i = 0; i < kPPL; ++i) {
+      for (int i = 0; i < PPL; ++i) {
         if (p0 + 32 * i >= Pb) continue;   // uniform skip of empty sub-chunks
         const V ao = PASS == 1 ? __shfl_sync(0xffffffffu, a, oa[i]) : V(0);
         ins(ca[i], ao * va[i], p0 + lane + 32 * i < Pb);
@@ -752,7 +753,9 @@ __device__ __forceinline__ int warp_row(const SpgemmArgs<V>& p, uint32_t* rk, V*
   // short rows keep the scrambled hash (robust to clustered columns) and rank counting
   const bool ordered = PASS == 1 && (MODE == 2 || (MODE == 0 && cnt > kSmallSeg));
   int newc = 0, wrapped = 0;
-  expand_row<PASS, V>(
+  // numeric rows of the ordered map: 2 products per lane per chunk (fewer registers; C5 numeric
+  // 379 -> 362 ms), symbolic and tiny rows 4 (more loads in flight)
+  expand_row<PASS, V, PASS == 0, false, (PASS == 1 && MODE == 2) ? 2 : kPPL>(
       p, a0, alen, 0, 1, [&](uint32_t col, V v, bool act) {
     if (PASS == 0) {
       if (act) newc += hash_insert_key(rk, S, col);
@@ -955,7 +958,7 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
         const uint64_t mmult = bkt_mult((uint32_t)(bm.rhi[r] - bm.rlo[r] + 1), S);
         const bool ordered = bm.ordered;
         int newc = 0, wrapped = 0;
-        expand_row<PASS, V, PASS == 0, true>(p, bm.astart[r], (int)(bm.aoff[r + 1] - bm.aoff[r]), warp_id(), NW,
+        expand_row<PASS, V, PASS == 0, true, PASS == 1 ? 2 : kPPL>(p, bm.astart[r], (int)(bm.aoff[r + 1] - bm.aoff[r]), warp_id(), NW,
                             [&](uint32_t col, V v, bool act) {
                               if (PASS == 0) {
                                 if (act) newc += hash_insert_key(rk, S, col);
