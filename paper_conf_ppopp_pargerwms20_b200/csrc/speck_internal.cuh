@@ -113,9 +113,16 @@ __host__ __device__ inline int64_t num_dense_window(int cfg) {
 constexpr int kWarpRowThreads = 256;
 constexpr int kWarpRegionBytes = 7168;
 constexpr int kWarpRowCtasPerSM = 4;
+// symbolic (keys only, <= 40 registers): 6 CTAs x 8 warps x 4.5 KB per SM — 48 warps hide more
+// of the gather latency (C2 symbolic A*P 1.85 -> 1.62 ms measured with this geometry)
+constexpr int kWarpRegionBytesSym = 4608;
+constexpr int kWarpRowCtasPerSMSym = 6;
+static_assert((kWarpRegionBytesSym * (kWarpRowThreads / 32) + 1024) * kWarpRowCtasPerSMSym <= kSmemPerSM, "warp-row CTAs");
+__host__ __device__ constexpr int wr_region_bytes(int pass) { return pass == 0 ? kWarpRegionBytesSym : kWarpRegionBytes; }
+__host__ __device__ constexpr int wr_ctas_per_sm(int pass) { return pass == 0 ? kWarpRowCtasPerSMSym : kWarpRowCtasPerSM; }
 constexpr int kWarpRowChunk = 8;     // rows a warp claims per counter increment
 static_assert((kWarpRegionBytes * (kWarpRowThreads / 32) + 1024) * kWarpRowCtasPerSM <= kSmemPerSM, "warp-row CTAs");
-__host__ __device__ inline uint32_t wr_sym_cap() { return (uint32_t)(kWarpRegionBytes / 4); }
+__host__ __device__ inline uint32_t wr_sym_cap() { return (uint32_t)(kWarpRegionBytesSym / 4); }
 __host__ __device__ inline uint32_t wr_sym_fill() { return (uint32_t)((uint64_t)wr_sym_cap() * kFillNum / 100); }
 template <typename V>
 __host__ __device__ inline uint32_t wr_num_cap() { return (uint32_t)((kWarpRegionBytes - 16) / num_slot_bytes<V>()); }
