@@ -227,12 +227,12 @@ def run_speck(args):
         # balanced product split (Alg. 1 on the replicated A; identical on every rank) — untimed
         bnds = []
         (_, A0, B0) = probs[0]
-        bnds.append(sdist.partition_rows(handles[0].row_analysis(A0, B0)[0], world))
+        bnds.append(sdist.partition_rows(handles[0].row_products(A0, B0), world))
         if cfg == "c2":
             # the second product's A is R; its B (AP) has the same row structure on every rank
             (_, R, _) = probs[1]
             AP0 = handles[0].spgemm(A0, B0)
-            bnds.append(sdist.partition_rows(handles[1].row_analysis(R, AP0)[0], world))
+            bnds.append(sdist.partition_rows(handles[1].row_products(R, AP0), world))
             del AP0
         state["bounds"] = bnds
 

@@ -146,6 +146,21 @@ speck_status_t speck_row_analysis(speck_handle_t handle, const speck_csr_t* A, c
                                   int64_t* prods, int32_t* maxlen, int32_t* colmin, int32_t* colmax,
                                   speck_stream_t stream);
 
+/* Row analysis restricted to the product counts (Alg. 1 line 10):
+ *   prods[i] = Σ_{k ∈ A_i} |B_k|, device int64 [A.rows], caller-owned.
+ * The multi-GPU partitioner's balanced row split.  Asynchronous. */
+speck_status_t speck_row_products(speck_handle_t handle, const speck_csr_t* A, const speck_csr_t* B, int64_t* prods,
+                                  speck_stream_t stream);
+
+/* Workspace allocator hooks (e.g. the PyTorch caching allocator): alloc(bytes, stream, ctx)
+ * returns device memory usable on `stream` (NULL on failure -> SPECK_ERR_OUT_OF_MEMORY),
+ * release(p, stream, ctx) gives it back.  Without hooks the handle uses cudaMallocAsync /
+ * cudaFreeAsync.  Setting (or clearing, with NULLs) the hooks first releases the handle's
+ * current workspace, so call it before speck_analyze; a pending speck_spgemm must be complete. */
+typedef void* (*speck_alloc_fn)(size_t bytes, speck_stream_t stream, void* ctx);
+typedef void (*speck_release_fn)(void* ptr, speck_stream_t stream, void* ctx);
+speck_status_t speck_set_allocator(speck_handle_t handle, speck_alloc_fn alloc, speck_release_fn release, void* ctx);
+
 /* Statistics of the last analyze/spgemm (host struct). */
 speck_status_t speck_get_stats(speck_handle_t handle, speck_stats_t* out);
 

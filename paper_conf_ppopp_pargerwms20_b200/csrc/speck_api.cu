@@ -71,6 +71,10 @@ struct speck_handle_s {
   int seg_shift = 15, nchunks = 0;
   int64_t long_thr = INT64_MAX, n_cand = 0, n_segs = 0, cand_start = 0;
   Buf chunk_cnt, cand, nseg, seg_off, segs;
+  // user workspace allocator (speck_set_allocator)
+  speck_alloc_fn ualloc = nullptr;
+  speck_release_fn urelease = nullptr;
+  void* uctx = nullptr;
 };
 
 namespace {
@@ -104,12 +108,25 @@ speck_status_t fail(speck_handle_t h, speck_status_t s, const char* fmt, ...) {
                   __FILE__, __LINE__);                                                                \
   } while (0)
 
-speck_status_t ensure(speck_handle_t h, Buf& b, size_t bytes, cudaStream_t s, bool exact = false) {
-  if (bytes <= b.cap) return SPECK_OK;
-  if (b.p) CK(cudaFreeAsync(b.p, s));
+void release_buf(speck_handle_t h, Buf& b, cudaStream_t s) {
+  if (b.p) {
+    if (h->urelease) h->urelease(b.p, static_cast<speck_stream_t>(s), h->uctx);
+    else cudaFreeAsync(b.p, s);
+  }
   b.p = nullptr;
   b.cap = 0;
+}
+
+speck_status_t ensure(speck_handle_t h, Buf& b, size_t bytes, cudaStream_t s, bool exact = false) {
+  if (bytes <= b.cap) return SPECK_OK;
+  release_buf(h, b, s);
   size_t want = std::max<size_t>(exact ? bytes : bytes + bytes / 4, 4096);
+  if (h->ualloc) {
+    b.p = h->ualloc(want, static_cast<speck_stream_t>(s), h->uctx);
+    if (!b.p) return fail(h, SPECK_ERR_OUT_OF_MEMORY, "workspace allocation of %zu bytes failed (user allocator)", want);
+    b.cap = want;
+    return SPECK_OK;
+  }
   cudaError_t e = cudaMallocAsync(&b.p, want, s);
   if (e != cudaSuccess) {
     (void)cudaGetLastError();
@@ -854,8 +871,11 @@ speck_status_t speck_destroy(speck_handle_t h) {
   Buf* bufs[] = {&h->prods, &h->maxlen, &h->colmin, &h->colmax, &h->cnt, &h->hist, &h->hist_off, &h->bins, &h->stats,
                  &h->scan_status, &h->resume, &h->small, &h->ana_long, &h->chunk_cnt, &h->cand, &h->nseg,
                  &h->seg_off, &h->segs, &h->bm_pool, &h->bm_off};
-  for (Buf* b : bufs)
-    if (b->p) cudaFree(b->p);
+  for (Buf* b : bufs) {
+    if (!b->p) continue;
+    if (h->urelease) h->urelease(b->p, nullptr, h->uctx);
+    else cudaFree(b->p);
+  }
   if (h->h_pinned) cudaFreeHost(h->h_pinned);
   for (int i = 0; i < kMaxStreams; ++i) {
     if (h->streams[i]) cudaStreamDestroy(h->streams[i]);
@@ -959,6 +979,34 @@ speck_status_t speck_row_analysis(speck_handle_t h, const speck_csr_t* A, const 
   st = run_analysis(h, A, B, pr, maxlen, colmin, colmax, nullptr, s);
   cudaSetDevice(prev);
   return st;
+}
+
+speck_status_t speck_row_products(speck_handle_t h, const speck_csr_t* A, const speck_csr_t* B, int64_t* prods,
+                                  speck_stream_t stream) {
+  if (!h) return SPECK_ERR_INVALID_ARGUMENT;
+  if (!prods && A && A->rows > 0) return fail(h, SPECK_ERR_INVALID_ARGUMENT, "prods is NULL");
+  return speck_row_analysis(h, A, B, prods, nullptr, nullptr, nullptr, stream);
+}
+
+speck_status_t speck_set_allocator(speck_handle_t h, speck_alloc_fn alloc, speck_release_fn release, void* ctx) {
+  if (!h) return SPECK_ERR_INVALID_ARGUMENT;
+  if ((alloc == nullptr) != (release == nullptr))
+    return fail(h, SPECK_ERR_INVALID_ARGUMENT, "alloc and release must both be set or both be NULL");
+  int prev = 0;
+  cudaGetDevice(&prev);
+  cudaSetDevice(h->device);
+  cudaDeviceSynchronize();   // no kernel may still use the workspace being released
+  Buf* bufs[] = {&h->prods, &h->maxlen, &h->colmin, &h->colmax, &h->cnt, &h->hist, &h->hist_off, &h->bins, &h->stats,
+                 &h->scan_status, &h->resume, &h->small, &h->ana_long, &h->chunk_cnt, &h->cand, &h->nseg,
+                 &h->seg_off, &h->segs, &h->bm_pool, &h->bm_off};
+  for (Buf* b : bufs) release_buf(h, *b, nullptr);
+  cudaStreamSynchronize(nullptr);
+  h->ualloc = alloc;
+  h->urelease = release;
+  h->uctx = ctx;
+  h->analyzed = false;
+  cudaSetDevice(prev);
+  return SPECK_OK;
 }
 
 speck_status_t speck_get_stats(speck_handle_t h, speck_stats_t* out) {

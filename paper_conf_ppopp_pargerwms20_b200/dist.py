@@ -78,7 +78,7 @@ def _default_local(A, B):
 
 def _default_prods(A, B):
     from .speck import default_handle
-    return default_handle(A.row_ptr.device.index).row_analysis(A, B)[0]
+    return default_handle(A.row_ptr.device.index).row_products(A, B)
 
 
 def broadcast_csr(M, src: int = 0, group=None, device=None):

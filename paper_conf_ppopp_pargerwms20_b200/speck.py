@@ -34,8 +34,10 @@ STATUS = {
 EXPORTS = [
     "speck_create", "speck_destroy", "speck_set_option", "speck_analyze", "speck_spgemm", "speck_row_analysis",
     "speck_get_stats", "speck_status_string", "speck_last_error", "speck_version", "speck_block_merge",
-    "speck_group_size", "speck_hash_probe", "speck_exclusive_scan",
+    "speck_group_size", "speck_hash_probe", "speck_exclusive_scan", "speck_row_products", "speck_set_allocator",
 ]
+_ALLOC_FN = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p, ctypes.c_void_p)
+_RELEASE_FN = ctypes.CFUNCTYPE(None, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p)
 
 
 class SpeckError(RuntimeError):
@@ -95,6 +97,8 @@ def load() -> ctypes.CDLL:
         L.speck_group_size.argtypes = [P, I32, P, P, P, I64, P, P]
         L.speck_hash_probe.argtypes = [P, P, P, I64, I32, P, P, P]
         L.speck_exclusive_scan.argtypes = [P, P, I64, P, P]
+        L.speck_row_products.argtypes = [P, ctypes.POINTER(_Csr), ctypes.POINTER(_Csr), P, P]
+        L.speck_set_allocator.argtypes = [P, _ALLOC_FN, _RELEASE_FN, P]
         for f in EXPORTS:
             if f not in ("speck_status_string", "speck_last_error", "speck_version"):
                 getattr(L, f).restype = ctypes.c_int
@@ -154,7 +158,7 @@ def _ptr(t: Optional[torch.Tensor]):
 class Handle:
     """A libspeck handle (workspace + plan state), bound to one CUDA device."""
 
-    def __init__(self, device: Optional[int] = None, **options):
+    def __init__(self, device: Optional[int] = None, torch_allocator: bool = True, **options):
         self._L = load()
         self.device = torch.cuda.current_device() if device is None else int(device)
         h = ctypes.c_void_p()
@@ -162,11 +166,33 @@ class Handle:
         if st != 0:
             raise SpeckError(st, "speck_create failed (is a CUDA device available?)")
         self._h = h
+        if torch_allocator:
+            self.use_torch_allocator()
         for k, v in options.items():
             self.set_option(k, v)
 
+    def use_torch_allocator(self):
+        """Route the handle's workspace through PyTorch's caching allocator (speck_set_allocator)."""
+        dev = self.device
+
+        def _alloc(nbytes, stream, ctx):
+            try:
+                return torch.cuda.caching_allocator_alloc(int(nbytes), dev, stream or 0)
+            except RuntimeError:
+                return None
+
+        def _release(ptr, stream, ctx):
+            torch.cuda.caching_allocator_delete(ptr)
+
+        self._alloc_cb, self._release_cb = _ALLOC_FN(_alloc), _RELEASE_FN(_release)   # keep alive
+        self._check(self._L.speck_set_allocator(self._h, self._alloc_cb, self._release_cb, None))
+
     def close(self):
         if getattr(self, "_h", None):
+            import sys
+            if getattr(self, "_alloc_cb", None) is not None and sys.is_finalizing():
+                self._h = None   # interpreter teardown: torch's allocator may be gone; the process frees all
+                return
             self._L.speck_destroy(self._h)
             self._h = None
 
@@ -208,6 +234,13 @@ class Handle:
         val = torch.empty(nnz, dtype=A.val.dtype, device=dev)
         self.numeric(A, B, rp, col, val, stream=stream)
         return CSR(A.rows, B.cols, rp, col, val)
+
+    def row_products(self, A, B, stream=None) -> torch.Tensor:
+        """Alg. 1 line 10 per row: products int64 device tensor (speck_row_products)."""
+        prods = torch.empty(A.rows, dtype=torch.int64, device=A.row_ptr.device)
+        self._check(self._L.speck_row_products(self._h, ctypes.byref(_csr(A)), ctypes.byref(_csr(B)),
+                                               prods.data_ptr(), _stream(stream)))
+        return prods
 
     def row_analysis(self, A, B, stream=None):
         """Alg. 1 per row: (prods int64, maxlen int32, colmin int32, colmax int32) device tensors."""

@@ -286,6 +286,30 @@ def test_very_long_rows_of_a(dev, dt):
     assert_parity(A, B, C)
 
 
+def test_row_products_and_allocators(dev):
+    """speck_row_products equals Alg. 1's products (oracle); the result is the same whether the
+    workspace comes from cudaMallocAsync or from PyTorch's caching allocator (speck_set_allocator)."""
+    A = W.rmat(11, 16, seed=41, dtype=torch.float32)
+    want = oracle.row_analysis(A, A)[0]
+    Ad = A.to(dev)
+    for ta in (True, False):
+        h = sp.Handle(0, torch_allocator=ta)
+        got = h.row_products(Ad, Ad).cpu().numpy()
+        assert np.array_equal(got, want)
+        C = h.spgemm(Ad, Ad)
+        torch.cuda.synchronize()
+        assert_parity(A, A, C)
+        h.close()
+    # switching the allocator on a used handle releases the old workspace and keeps working
+    h = sp.Handle(0, torch_allocator=False)
+    C1 = h.spgemm(Ad, Ad)
+    h.use_torch_allocator()
+    C2 = h.spgemm(Ad, Ad)
+    torch.cuda.synchronize()
+    assert torch.equal(C1.col, C2.col) and torch.equal(C1.row_ptr, C2.row_ptr)
+    h.close()
+
+
 def test_fig5_dense_window_of_three(dev):
     """Fig. 5: one row, 6 columns, window 3, products at c0,c2,c4,c4,c5 -> c0=1 c2=1 c4=2 c5=1."""
     kv, _ = golden("fig5_dense.txt")
