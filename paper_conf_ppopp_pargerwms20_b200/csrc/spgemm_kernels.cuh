@@ -162,12 +162,16 @@ __device__ __forceinline__ int warp_write_ordered(const uint32_t* rk, const V* r
     const uint32_t mine = occ & (w1 - c0 >= 32 ? 0xffffffffu : ((1u << (w1 - c0)) - 1u));
     // fast path (warp-uniform): no full bucket in the window and no run entering it, so every
     // run is its bucket: rank among the bucket's 8 keys by shuffles, no divergent walk
-    const uint32_t fullb = occ & (occ >> 1) & (occ >> 2) & (occ >> 3) & (occ >> 4) & (occ >> 5) & (occ >> 6) & (occ >> 7) &
-                           0x01010101u;
+    const uint32_t fullb = __vcmpeq4(occ, 0xffffffffu);   // 0xff in every byte (bucket) that is full
     if (!fullb && carry == 0) {
+      // rank among the bucket's 8 keys: two 16-byte loads shared by the bucket's 8 lanes
+      uint32_t q[8];
+      const uint32_t a = (uint32_t)__cvta_generic_to_shared(rk + c0 + (lane & ~7));
+      asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(q[0]), "=r"(q[1]), "=r"(q[2]), "=r"(q[3]) : "r"(a));
+      asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(q[4]), "=r"(q[5]), "=r"(q[6]), "=r"(q[7]) : "r"(a + 16));
       int rank = 0;
 #pragma unroll
-      for (int d = 1; d < 8; ++d) rank += __shfl_sync(0xffffffffu, k, (lane & ~7) | ((lane + d) & 7)) < k;
+      for (int d = 0; d < 8; ++d) rank += q[d] < k;
       if ((mine >> lane) & 1u) {
         const int64_t o = ob + before + written + __popc(occ & ((1u << (lane & ~7)) - 1u)) + rank;
         C_col[o] = (int32_t)k;
