@@ -296,11 +296,19 @@ __device__ void block_write_ordered(const uint32_t* rk, const V* rv, uint32_t S,
   const int lane = lane_id(), wp = warp_id();
   const uint32_t SW = ((S + NW - 1) / NW + 31u) & ~31u;
   const uint32_t w0 = min(S, wp * SW), w1 = min(S, w0 + SW);
+  // occupancy of the warp's range: 4 slots per lane per 16-byte load
   int cw = 0;
-  for (uint32_t c0 = w0; c0 < w1; c0 += 32) {
-    const uint32_t s = c0 + lane;
-    cw += __popc(__ballot_sync(0xffffffffu, s < w1 && rk[s] != kEmptyKey));
+  for (uint32_t c = w0 + 4 * lane; c < w1; c += 128) {
+    if (c + 4 <= w1) {
+      uint32_t q0, q1, q2, q3;
+      asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(q0), "=r"(q1), "=r"(q2), "=r"(q3)
+                   : "r"((uint32_t)__cvta_generic_to_shared(rk + c)));
+      cw += (q0 != kEmptyKey) + (q1 != kEmptyKey) + (q2 != kEmptyKey) + (q3 != kEmptyKey);
+    } else {
+      for (uint32_t t = c; t < w1; ++t) cw += rk[t] != kEmptyKey;
+    }
   }
+  cw = warp_sum(cw);
   if (lane == 0) part[wp] = cw;
   __syncthreads();
   int before = 0;
