@@ -18,6 +18,11 @@ sample of the same workload (there is no reference code to install: the referenc
 from __future__ import annotations
 
 import argparse
+import os as _os
+
+# the largest configurations allocate C of 70-90 GB next to large workspaces: let PyTorch's
+# caching allocator grow segments instead of fragmenting (user settings take precedence)
+_os.environ.setdefault("PYTORCH_CUDA_ALLOC_CONF", "expandable_segments:True")
 import json
 import os
 import statistics
@@ -148,22 +153,26 @@ def run_oracle_sample(cfg, probs_host, budget_s=20.0, threads=None):
     (_, A, B), = probs_host
     prods = oracle.row_analysis(A, B)[0]
     total = int(prods.sum())
-    # contiguous row block sized for ~budget_s at ~0.15 G products/s/thread
-    rate = 0.15e9 * oracle.num_threads()
-    want = min(total, int(budget_s * rate))
-    if want >= total:
-        r0, r1 = 0, A.rows
-    else:
-        pre = np.cumsum(prods)
-        start = A.rows // 3
-        base = pre[start - 1] if start > 0 else 0
-        r1 = int(np.searchsorted(pre, base + want)) + 1
-        r0, r1 = start, min(max(r1, start + 1), A.rows)
-    sp = int(prods[r0:r1].sum())
-    t0 = time.perf_counter()
-    oracle.spgemm(A, B, r0, r1, with_scale=False)
-    t = time.perf_counter() - t0
-    return 2 * sp / t / 1e9, t, sp, f"rows [{r0},{r1}) of {A.rows} ({sp} of {total} products)"
+    # consecutive row blocks from A.rows // 3 on, each <= ORACLE_BLOCK_PRODUCTS products (the
+    # oracle materialises its block's C on the host: C3/C5 are 70-90 GB), until ~budget_s of
+    # CPU work or the end of the matrix
+    pre = np.cumsum(prods)
+    r0 = start = 0 if total <= ORACLE_BLOCK_PRODUCTS else A.rows // 3
+    t = 0.0
+    sp = 0
+    while r0 < A.rows and t < budget_s:
+        base = pre[r0 - 1] if r0 > 0 else 0
+        r1 = min(max(int(np.searchsorted(pre, base + ORACLE_BLOCK_PRODUCTS, side="right")), r0 + 1), A.rows)
+        t0 = time.perf_counter()
+        out = oracle.spgemm(A, B, r0, r1, with_scale=False)
+        t += time.perf_counter() - t0
+        del out
+        sp += int(prods[r0:r1].sum())
+        r0 = r1
+    return 2 * sp / t / 1e9, t, sp, f"rows [{start},{r0}) of {A.rows} ({sp} of {total} products)"
+
+
+ORACLE_BLOCK_PRODUCTS = 200_000_000
 
 
 # --------------------------------------------------------------------------- speck arm
@@ -326,6 +335,11 @@ def run_speck(args):
     # ---- end-to-end through the public API with host buffers (rank 0, N=1)
     e2e = None
     if not args.no_e2e:
+        # free the timed loop's result and workspaces first (C3/C5: C is 70-90 GB)
+        state["out"] = None
+        for h in handles:
+            h.close()
+        torch.cuda.empty_cache()
         e2e = run_e2e(sp, probs, dev, min(args.steps, 5), step_products, compute, world)
 
     # ---- CPU baseline: the oracle on this host's cores (rank 0, N=1)
@@ -365,6 +379,9 @@ def run_speck(args):
         dist.destroy_process_group()
 
 
+E2E_STAGING_BYTES = 2 << 30
+
+
 def run_e2e(sp, probs, dev, steps, step_products, compute, world):
     """Same metric through the public API, host (pinned) inputs in, host result out.  At N>1
     every rank copies the replicated inputs and reads back its own row block of the result;
@@ -381,7 +398,7 @@ def run_e2e(sp, probs, dev, steps, step_products, compute, world):
     bi = sum(t.numel() * t.element_size() for pair in host_in for M in pair if M is not None
              for t in (M.row_ptr, M.col, M.val))
     stream = torch.cuda.current_stream()
-    times, bo = [], 0
+    times, bo, res = [], 0, None
     for it in range(steps + 1):
         torch.cuda.synchronize()
         if world > 1:
@@ -396,12 +413,20 @@ def run_e2e(sp, probs, dev, steps, step_products, compute, world):
                 Md.col.copy_(Mh.col, non_blocking=True)
                 Md.val.copy_(Mh.val, non_blocking=True)
         C = compute(dev_in, h)[-1]
-        res = [torch.empty(t.shape, dtype=t.dtype, pin_memory=True) for t in (C.row_ptr, C.col, C.val)]
-        for r, t in zip(res, (C.row_ptr, C.col, C.val)):
-            r.copy_(t, non_blocking=True)
+        outs = [t.view(torch.uint8) for t in (C.row_ptr, C.col, C.val) if t.numel()]
+        if res is None:                                # first (untimed) iteration: pinned staging buffer
+            # the result is streamed through a bounded pinned buffer (C3/C5 results are 70-90 GB,
+            # more than the host can pin); every byte of C still crosses PCIe/C2C each step
+            res = torch.empty(min(sum(t.numel() for t in outs), E2E_STAGING_BYTES), dtype=torch.uint8,
+                              pin_memory=True)
+        for t in outs:
+            for o in range(0, t.numel(), res.numel()):
+                n = min(res.numel(), t.numel() - o)
+                res[:n].copy_(t[o:o + n], non_blocking=True)
         b.record(stream)
         torch.cuda.synchronize()
-        bo = sum(r.numel() * r.element_size() for r in res)
+        bo = sum(t.numel() for t in outs)
+        del C, outs                                    # the next step's C must not coexist with this one
         if it > 0:                                     # first iteration warms the handles
             times.append(a.elapsed_time(b))
     ms = statistics.mean(times)
