@@ -66,7 +66,12 @@ struct SegPlanArgs {
   int64_t bitmap_cols;     // >0: rows whose column range fits are done by k_long_bitmap (no segments)
   const uint32_t* bm_pool; // bitmaps kept by the symbolic step (SpgemmArgs::bm_pool), or null
   const int64_t* bm_off;   // per candidate: word offset in bm_pool, -1 = rebuild
+  int split_max;           // >1: CTAs per candidate; rows with a kept bitmap split their A entries
+                           //     over up to this many CTAs (C.val zeroed beforehand by the host)
 };
+constexpr int64_t kSplitProducts = 1 << 19;   // products per CTA of a split long row
+constexpr int kSplitPieces = 8;               // CTAs per candidate when splitting
+constexpr int64_t kSplitMaxCand = 4096;       // split only with few candidates (grid = candidates x pieces)
 
 // Long rows whose column range fits the shared-memory bitmap of k_long_bitmap.
 __device__ __forceinline__ bool bitmap_row(const SegPlanArgs& a, int32_t row) {
@@ -271,9 +276,20 @@ __global__ void __launch_bounds__(kBitmapThreads, 1) k_long_bitmap(SpgemmArgs<V>
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ int64_t part[NW + 1];
   __shared__ LongList<V> longs;
-  const int32_t row = a.cand[blockIdx.x];
+  const int ci = blockIdx.x / a.split_max, piece = blockIdx.x % a.split_max;
+  const int32_t row = a.cand[ci];
   const int64_t ob = a.C_rp[row], cnt = a.C_rp[row + 1] - ob;
   if (cnt <= a.limit || !bitmap_row(a, row)) return;
+  const long long bmo = a.bm_pool ? a.bm_off[ci] : -1ll;
+  // giant rows whose bitmap was kept (the structure needs no cross-CTA merge): the row's A
+  // entries are split over `pieces` CTAs, each adding its products' values (C4: 64 rows of 4M
+  // products were the numeric step's critical path on 64 SMs)
+  int pieces = 1;
+  if (bmo >= 0 && a.split_max > 1) {
+    const int64_t want = p.prods[row] / kSplitProducts;
+    pieces = want < 1 ? 1 : (want > a.split_max ? a.split_max : (int)want);
+  }
+  if (piece >= pieces) return;
   const int tid = threadIdx.x, lane = lane_id(), wp = warp_id();
   const uint32_t lo = (uint32_t)a.colmin[row] & ~31u;
   const int W = (int)(((int64_t)a.colmax[row] + 1 - lo + 31) / 32);
@@ -281,9 +297,10 @@ __global__ void __launch_bounds__(kBitmapThreads, 1) k_long_bitmap(SpgemmArgs<V>
   uint32_t* bits = reinterpret_cast<uint32_t*>(smem);
   int32_t* gpre = reinterpret_cast<int32_t*>(smem + (size_t)G * 128);       // after 32*G words
   uint16_t* wpre = reinterpret_cast<uint16_t*>(smem + (size_t)G * 128 + (size_t)G * 4);
-  const int64_t a0 = p.A_rp[row];
-  const int alen = (int)(p.A_rp[row + 1] - a0);
-  const long long bmo = a.bm_pool ? a.bm_off[blockIdx.x] : -1ll;
+  const int64_t ar0 = p.A_rp[row];
+  const int arlen = (int)(p.A_rp[row + 1] - ar0);
+  const int64_t a0 = ar0 + (int64_t)arlen * piece / pieces;             // this CTA's slice of A_i
+  const int alen = (int)(ar0 + (int64_t)arlen * (piece + 1) / pieces - a0);
   if (bmo >= 0) {
     // the symbolic step kept this row's bitmap: load it instead of rebuilding it (pass 1)
     const uint32_t* src = a.bm_pool + bmo;
@@ -297,7 +314,7 @@ __global__ void __launch_bounds__(kBitmapThreads, 1) k_long_bitmap(SpgemmArgs<V>
   // pay 32x their A traffic that way: there hub rows of B (>= kLongB entries) go to a shared
   // list streamed by all warps and the other batches go round-robin over the warps.
   bool listed = false;
-  if (p.prods[row] < (int64_t)kAllAvgLen * alen) listed = collect_long_rows<1, V>(p, a0, alen, longs);
+  if (p.prods[row] < (int64_t)kAllAvgLen * arlen) listed = collect_long_rows<1, V>(p, a0, alen, longs);
   else __syncthreads();
   // 1. structure
   auto set_bit = [&](uint32_t col, V, bool act) {
@@ -335,7 +352,9 @@ __global__ void __launch_bounds__(kBitmapThreads, 1) k_long_bitmap(SpgemmArgs<V>
     // group's entries span few sectors), dense groups one word at a time across the warp
     const int mx = __reduce_max_sync(0xffffffffu, (unsigned)pc);
     const uint32_t cbase = lo + (uint32_t)g * 1024u;
-    if (mx <= 8) {
+    if (piece > 0) {
+      // another piece of a split row writes C.col
+    } else if (mx <= 8) {
       uint32_t wv = word;
       int o = run + excl;
       while (wv) {
@@ -355,7 +374,9 @@ __global__ void __launch_bounds__(kBitmapThreads, 1) k_long_bitmap(SpgemmArgs<V>
     run += __shfl_sync(0xffffffffu, incl, 31);
   }
   // zero the row's values (coalesced), then make the zeros visible to the block's atomics
-  for (int64_t i = tid; i < cnt; i += T) p.C_val[ob + i] = V(0);
+  // (split rows: C.val was zeroed before the launch)
+  if (pieces == 1)
+    for (int64_t i = tid; i < cnt; i += T) p.C_val[ob + i] = V(0);
   __syncthreads();
   // 3. values
   V* cv = p.C_val + ob;

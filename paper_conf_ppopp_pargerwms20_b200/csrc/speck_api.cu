@@ -386,6 +386,7 @@ SegPlanArgs seg_plan_args(speck_handle_t h, const int64_t* C_rp) {
   s.bitmap_cols = (h->opt_long_bitmap == 2 || (h->opt_long_bitmap && !s.prefer_parallel)) ? kBitmapMaxCols : 0;
   s.bm_pool = (h->bm_enabled && s.bitmap_cols > 0) ? static_cast<const uint32_t*>(h->bm_pool.p) : nullptr;
   s.bm_off = static_cast<const int64_t*>(h->bm_off.p);
+  s.split_max = 1;
   return s;
 }
 
@@ -432,13 +433,23 @@ speck_status_t run_pass(speck_handle_t h, int pass, int lb, const int64_t* cat_s
                                                            static_cast<Seg*>(h->segs.p));
     CKL();
   }
+  // few long rows with kept bitmaps: split them over several CTAs (zero C.val first, on the
+  // user stream, before any kernel of this pass writes it)
+  SegPlanArgs sa0{};
+  if (pass == 1 && h->seg_enabled && h->n_cand > 0) {
+    sa0 = seg_plan_args<V>(h, a.C_rp);
+    if (sa0.bitmap_cols > 0 && sa0.bm_pool && h->n_cand <= kSplitMaxCand) {
+      sa0.split_max = kSplitPieces;
+      CK(cudaMemsetAsync(a.C_val, 0, (size_t)h->nnz_c * sizeof(V), s));
+    }
+  }
   if ((st = fork(h, s, ns))) return st;
   int si = 0;
   const int32_t* bins = static_cast<const int32_t*>(h->bins.p);
   if (pass == 1 && h->seg_enabled && h->n_cand > 0) {
-    const SegPlanArgs sa = seg_plan_args<V>(h, a.C_rp);
+    const SegPlanArgs sa = sa0;
     if (sa.bitmap_cols > 0) {
-      k_long_bitmap<V><<<(unsigned)h->n_cand, kBitmapThreads, kCfgMapBytes[kNumCfg - 1], h->streams[si]>>>(a, sa);
+      k_long_bitmap<V><<<(unsigned)(h->n_cand * sa.split_max), kBitmapThreads, kCfgMapBytes[kNumCfg - 1], h->streams[si]>>>(a, sa);
       CKL();
       si = (si + 1) % ns;
     }

@@ -263,21 +263,22 @@ def test_bitmap_reuse(dev, reuse, dt):
     assert torch.equal(C2.col.cpu(), C.col.cpu())
 
 
+@pytest.mark.parametrize("alen_long", [20_000, 150_000])
 @pytest.mark.parametrize("dt", [torch.float32, torch.float64])
-def test_very_long_rows_of_a(dev, dt):
+def test_very_long_rows_of_a(dev, dt, alen_long):
     """C4-like: a few rows of A with 20k NZ (over 2^16 columns of B, rows of 8 entries, plus a few
     hub rows of 5000 entries) -> long rows of C handled by the bitmap CTA with the shared hub-row
     list (segments would binary-search every referenced B row per segment)."""
     import numpy as _np
     rng = _np.random.default_rng(23)
-    nb = 40_000
+    nb = 40_000 if alen_long <= 40_000 else 200_000
     lens = np.full(nb, 8)
     lens[rng.choice(nb, 20, replace=False)] = 5000
     rows = np.repeat(np.arange(nb), lens)
     bc = np.concatenate([np.sort(rng.choice(1 << 16, size=int(l), replace=False)) for l in lens])
     B = W.csr_from_coo(nb, 1 << 16, torch.tensor(rows), torch.tensor(bc), None, dtype=dt, seed=24)
     na = 40
-    alen = np.where(np.arange(na) < 4, 20_000, 8)
+    alen = np.where(np.arange(na) < 4, min(alen_long, nb), 8)   # 150k: > 2^19 products -> split CTAs
     ar = np.repeat(np.arange(na), alen)
     ac = np.concatenate([np.sort(rng.choice(nb, size=int(l), replace=False)) for l in alen])
     A = W.csr_from_coo(na, nb, torch.tensor(ar), torch.tensor(ac), None, dtype=dt, seed=25)
