@@ -17,13 +17,29 @@ namespace speck {
 // ------------------------------------------------------------------------------------
 constexpr int kAnaU = 4;   // NZ per lane per iteration of the analysis
 
+// Per row of B: {length, first column, last column, 0} (first = INT_MAX, last = -1 if empty),
+// one 16-byte record, so the analysis makes one random access per NZ of A instead of three
+// (the B.row_ptr pair and two B.col gathers).  Built when rows of B are referenced several times.
+__global__ void __launch_bounds__(256) k_brow_info(const int64_t* __restrict__ B_rp, const int32_t* __restrict__ B_col,
+                                                   int64_t k, int4* __restrict__ info) {
+  for (int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < k; r += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t b0 = B_rp[r], b1 = B_rp[r + 1];
+    int4 v;
+    v.x = (int)(b1 - b0);
+    v.y = b1 > b0 ? B_col[b0] : INT_MAX;
+    v.z = b1 > b0 ? B_col[b1 - 1] : -1;
+    v.w = 0;
+    info[r] = v;
+  }
+}
+
 template <int GA>
 __global__ void __launch_bounds__(256) k_analysis(const int64_t* __restrict__ A_rp, const int32_t* __restrict__ A_col,
                                                   const int64_t* __restrict__ B_rp, const int32_t* __restrict__ B_col,
                                                   int64_t m, int64_t* __restrict__ prods, int32_t* __restrict__ maxlen,
                                                   int32_t* __restrict__ colmin, int32_t* __restrict__ colmax,
                                                   AnalysisStats* st, int32_t* __restrict__ long_rows,
-                                                  unsigned int* n_long) {
+                                                  unsigned int* n_long, const int4* __restrict__ binfo) {
   const int sub = threadIdx.x % GA;
   constexpr int RPW = 32 / GA;  // rows per warp and iteration
   const int64_t gwarp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -49,6 +65,19 @@ __global__ void __launch_bounds__(256) k_analysis(const int64_t* __restrict__ A_
       int64_t b0[kAnaU], b1[kAnaU];
 #pragma unroll
       for (int u = 0; u < kAnaU; ++u) k[u] = q + u * GA < a1 ? A_col[q + u * GA] : -1;
+      if (binfo) {
+        int4 r[kAnaU];
+#pragma unroll
+        for (int u = 0; u < kAnaU; ++u) r[u] = k[u] >= 0 ? __ldg(binfo + k[u]) : make_int4(0, INT_MAX, -1, 0);
+#pragma unroll
+        for (int u = 0; u < kAnaU; ++u) {
+          p += r[u].x;
+          ml = max(ml, r[u].x);
+          cmin = min(cmin, r[u].y);
+          cmax = max(cmax, r[u].z);
+        }
+        continue;
+      }
 #pragma unroll
       for (int u = 0; u < kAnaU; ++u) {
         b0[u] = k[u] >= 0 ? B_rp[k[u]] : 0;

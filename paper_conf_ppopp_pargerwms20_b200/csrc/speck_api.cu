@@ -43,7 +43,7 @@ struct speck_handle_s {
   int64_t opt_lb_sym = -1, opt_lb_num = -1, opt_force_acc = 0, opt_dense_window = 0, opt_timing = 0, opt_validate = 0,
           opt_disable_direct = 0, opt_fixed_g = 0, opt_streams = 4;
   // workspace
-  Buf prods, maxlen, colmin, colmax, cnt, hist, hist_off, bins, stats, scan_status, resume, small, ana_long;
+  Buf prods, maxlen, colmin, colmax, cnt, hist, hist_off, bins, stats, scan_status, resume, small, ana_long, binfo;
   unsigned long long* h_pinned = nullptr;  // pinned readback area (64 x u64)
   cudaStream_t streams[kMaxStreams] = {};
   cudaEvent_t ev_fork = nullptr, ev_join[kMaxStreams] = {};
@@ -141,7 +141,7 @@ int64_t ws_bytes(speck_handle_t h) {
   return (int64_t)(h->prods.cap + h->maxlen.cap + h->colmin.cap + h->colmax.cap + h->cnt.cap + h->hist.cap +
                    h->hist_off.cap + h->bins.cap + h->stats.cap + h->scan_status.cap + h->resume.cap + h->small.cap +
                    h->ana_long.cap + h->chunk_cnt.cap + h->cand.cap + h->nseg.cap + h->seg_off.cap + h->segs.cap +
-                   h->bm_pool.cap + h->bm_off.cap);
+                   h->bm_pool.cap + h->bm_off.cap + h->binfo.cap);
 }
 
 speck_status_t check_csr(speck_handle_t h, const speck_csr_t* M, const char* name, bool need_values) {
@@ -173,11 +173,20 @@ speck_status_t run_analysis(speck_handle_t h, const speck_csr_t* A, const speck_
   unsigned* nlong = reinterpret_cast<unsigned*>(static_cast<char*>(h->small.p) + 640);
   int32_t* lrows = static_cast<int32_t*>(h->ana_long.p);
   CK(cudaMemsetAsync(nlong, 0, 4, s));
+  // rows of B referenced several times on average: one 16-byte record per row of B
+  const int4* binfo = nullptr;
+  if (B->rows > 0 && A->nnz > 4 * B->rows && B->rows < ((int64_t)1 << 31)) {
+    if ((r = ensure(h, h->binfo, (size_t)B->rows * 16, s))) return r;
+    binfo = static_cast<const int4*>(h->binfo.p);
+    const unsigned bg = (unsigned)std::max<int64_t>(1, std::min<int64_t>((B->rows + 255) / 256, (int64_t)h->num_sms * 16));
+    k_brow_info<<<bg, 256, 0, s>>>(B->row_ptr, B->col_idx, B->rows, const_cast<int4*>(binfo));
+    CKL();
+  }
   const int ga = pow2_clamp(m > 0 ? (double)A->nnz / (double)m / kAnaU : 1.0, 1, 32);   // GA*kAnaU ~ avg row
   const unsigned agrid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((m * ga + 255) / 256, (int64_t)h->num_sms * 8));
 #define SPECK_ANA(GA)                                                                                        \
   k_analysis<GA><<<agrid, 256, 0, s>>>(A->row_ptr, A->col_idx, B->row_ptr, B->col_idx, m, prods, maxlen, colmin, \
-                                       colmax, st, lrows, nlong)
+                                       colmax, st, lrows, nlong, binfo)
   switch (ga) {
     case 1: SPECK_ANA(1); break;
     case 2: SPECK_ANA(2); break;
@@ -881,7 +890,7 @@ speck_status_t speck_destroy(speck_handle_t h) {
   cudaDeviceSynchronize();
   Buf* bufs[] = {&h->prods, &h->maxlen, &h->colmin, &h->colmax, &h->cnt, &h->hist, &h->hist_off, &h->bins, &h->stats,
                  &h->scan_status, &h->resume, &h->small, &h->ana_long, &h->chunk_cnt, &h->cand, &h->nseg,
-                 &h->seg_off, &h->segs, &h->bm_pool, &h->bm_off};
+                 &h->seg_off, &h->segs, &h->bm_pool, &h->bm_off, &h->binfo};
   for (Buf* b : bufs) {
     if (!b->p) continue;
     if (h->urelease) h->urelease(b->p, nullptr, h->uctx);
@@ -1009,7 +1018,7 @@ speck_status_t speck_set_allocator(speck_handle_t h, speck_alloc_fn alloc, speck
   cudaDeviceSynchronize();   // no kernel may still use the workspace being released
   Buf* bufs[] = {&h->prods, &h->maxlen, &h->colmin, &h->colmax, &h->cnt, &h->hist, &h->hist_off, &h->bins, &h->stats,
                  &h->scan_status, &h->resume, &h->small, &h->ana_long, &h->chunk_cnt, &h->cand, &h->nseg,
-                 &h->seg_off, &h->segs, &h->bm_pool, &h->bm_off};
+                 &h->seg_off, &h->segs, &h->bm_pool, &h->bm_off, &h->binfo};
   for (Buf* b : bufs) release_buf(h, *b, nullptr);
   cudaStreamSynchronize(nullptr);
   h->ualloc = alloc;
