@@ -387,8 +387,8 @@ __device__ __forceinline__ void expand_row(const SpgemmArgs<V>& p, int64_t a0, i
   const int c_step = share ? G : 1;
   int rot = 0;   // ALL: warp taking the next chunk (warp-uniform, identical in every warp)
   auto my_first = [&](int nsub) {   // ALL: first chunk of this warp among nsub, then advance the rotation
-    const int j0 = (wi - rot + nw) % nw;
-    rot = (rot + nsub) % nw;
+    const int j0 = (wi - rot) & (nw - 1);   // nw is a power of two (warps per CTA)
+    rot = (rot + nsub) & (nw - 1);
     return j0;
   };
   for (int b = b_first; b < nb; b += b_step) {
@@ -530,8 +530,8 @@ __device__ __forceinline__ void expand_long_list(const SpgemmArgs<V>& p, const L
     const int64_t s0 = L.bst[r];
     const V ao = L.a[r];
     const int nsub = (len + CH - 1) / CH;
-    const int j0 = (wi - rot + nw) % nw;
-    rot = (rot + nsub) % nw;
+    const int j0 = (wi - rot) & (nw - 1);   // nw is a power of two (warps per CTA)
+    rot = (rot + nsub) & (nw - 1);
     for (int q0 = j0 * CH; q0 < len; q0 += nw * CH) {
       uint32_t c[kPPL];
       V bv[kPPL];
