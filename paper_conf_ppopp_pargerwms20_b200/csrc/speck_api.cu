@@ -240,7 +240,7 @@ speck_status_t set_smem_attrs(speck_handle_t h) {
   CK(cudaFuncSetAttribute(k_long_bitmap<V>, cudaFuncAttributeMaxDynamicSharedMemorySize, kCfgMapBytes[kNumCfg - 1]));
   CK(cudaFuncSetAttribute(k_warp_rows<0, V, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytesSym * (kWarpRowThreads / 32)));
   CK(cudaFuncSetAttribute(k_warp_rows<1, V, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytes * (kWarpRowThreads / 32)));
-  CK(cudaFuncSetAttribute(k_warp_rows<1, V, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytes * (kWarpRowThreads / 32)));
+  CK(cudaFuncSetAttribute(k_warp_rows<1, V, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytesTiny * (kWarpRowThreads / 32)));
   CK(cudaFuncSetAttribute(k_warp_rows<1, V, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytes * (kWarpRowThreads / 32)));
   return SPECK_OK;
 }
@@ -285,8 +285,9 @@ speck_status_t launch_warp_rows(speck_handle_t h, int pass, const SpgemmArgs<V>&
   unsigned long long* ctr =
       reinterpret_cast<unsigned long long*>(static_cast<char*>(h->small.p) + 1024 + 8 * (pass == 0 ? 0 : 1 + mode));
   CK(cudaMemsetAsync(ctr, 0, 8, s));
-  const int64_t grid = std::min<int64_t>((a.n_entries + 7) / 8, (int64_t)h->num_sms * wr_ctas_per_sm(pass));
-  const size_t smem = (size_t)wr_region_bytes(pass) * (kWarpRowThreads / 32);
+  const int md = pass == 0 ? 0 : mode;
+  const int64_t grid = std::min<int64_t>((a.n_entries + 7) / 8, (int64_t)h->num_sms * wr_ctas_per_sm(pass, md));
+  const size_t smem = (size_t)wr_region_bytes(pass, md) * (kWarpRowThreads / 32);
   if (pass == 0) k_warp_rows<0, V, 0><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
   else if (mode == 1) k_warp_rows<1, V, 1><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
   else if (mode == 2) k_warp_rows<1, V, 2><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);

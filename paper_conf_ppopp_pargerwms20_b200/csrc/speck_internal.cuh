@@ -118,16 +118,27 @@ constexpr int kWarpRowCtasPerSM = 4;
 constexpr int kWarpRegionBytesSym = 4608;
 constexpr int kWarpRowCtasPerSMSym = 6;
 static_assert((kWarpRegionBytesSym * (kWarpRowThreads / 32) + 1024) * kWarpRowCtasPerSMSym <= kSmemPerSM, "warp-row CTAs");
-__host__ __device__ constexpr int wr_region_bytes(int pass) { return pass == 0 ? kWarpRegionBytesSym : kWarpRegionBytes; }
-__host__ __device__ constexpr int wr_ctas_per_sm(int pass) { return pass == 0 ? kWarpRowCtasPerSMSym : kWarpRowCtasPerSM; }
+// numeric tiny rows (<= kTinyCnt entries, MODE 1): 2 KB regions hold 2.5x 64 entries, so the
+// smem no longer caps the CTAs; 5 CTAs (40 warps, 48 registers) measured best (C2 numeric A*P
+// 2.64 -> 2.56 ms; 6 CTAs at 40 registers spill and lose: 2.61 ms; ty_* runs, round 1)
+constexpr int kWarpRegionBytesTiny = 2048;
+constexpr int kWarpRowCtasPerSMTiny = 5;
+static_assert((kWarpRegionBytesTiny * (kWarpRowThreads / 32) + 1024) * kWarpRowCtasPerSMTiny <= kSmemPerSM, "warp-row CTAs");
+__host__ __device__ constexpr int wr_region_bytes(int pass, int mode = 0) {
+  return pass == 0 ? kWarpRegionBytesSym : mode == 1 ? kWarpRegionBytesTiny : kWarpRegionBytes;
+}
+__host__ __device__ constexpr int wr_ctas_per_sm(int pass, int mode = 0) {
+  return pass == 0 ? kWarpRowCtasPerSMSym : mode == 1 ? kWarpRowCtasPerSMTiny : kWarpRowCtasPerSM;
+}
 constexpr int kWarpRowChunk = 8;     // rows a warp claims per counter increment
 static_assert((kWarpRegionBytes * (kWarpRowThreads / 32) + 1024) * kWarpRowCtasPerSM <= kSmemPerSM, "warp-row CTAs");
 __host__ __device__ inline uint32_t wr_sym_cap() { return (uint32_t)(kWarpRegionBytesSym / 4); }
 __host__ __device__ inline uint32_t wr_sym_fill() { return (uint32_t)((uint64_t)wr_sym_cap() * kFillNum / 100); }
 template <typename V>
-__host__ __device__ inline uint32_t wr_num_cap() { return (uint32_t)((kWarpRegionBytes - 16) / num_slot_bytes<V>()); }
+__host__ __device__ constexpr uint32_t wr_num_cap(int bytes = kWarpRegionBytes) { return (uint32_t)((bytes - 16) / num_slot_bytes<V>()); }
 template <typename V>
-__host__ __device__ inline uint32_t wr_num_val_offset() { return (wr_num_cap<V>() * 4u + 15u) & ~15u; }
+__host__ __device__ constexpr uint32_t wr_num_val_offset(int bytes = kWarpRegionBytes) { return (wr_num_cap<V>(bytes) * 4u + 15u) & ~15u; }
+static_assert(wr_num_cap<double>(kWarpRegionBytesTiny) >= (uint32_t)(kTinyCnt * 5 / 2), "tiny region holds 2.5x kTinyCnt");
 template <typename V>
 __host__ __device__ inline uint32_t wr_num_fill() { return (uint32_t)((uint64_t)wr_num_cap<V>() * kFillOrdered / 100); }
 

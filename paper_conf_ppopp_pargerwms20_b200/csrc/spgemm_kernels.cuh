@@ -1135,14 +1135,15 @@ __device__ __noinline__ void dense_row(const SpgemmArgs<V>& p, BlockMeta& bm, in
 // load balancing, every row of A (p.rows == nullptr).
 // -----------------------------------------------------------------------------------
 template <int PASS, typename V, int MODE>
-__global__ void __launch_bounds__(kWarpRowThreads, wr_ctas_per_sm(PASS))
+__global__ void __launch_bounds__(kWarpRowThreads, wr_ctas_per_sm(PASS, MODE))
     k_warp_rows(SpgemmArgs<V> p, unsigned long long* __restrict__ counter) {
   extern __shared__ __align__(16) unsigned char smem[];
   const int lane = lane_id();
-  unsigned char* region = smem + warp_id() * wr_region_bytes(PASS);
+  constexpr int kRegion = wr_region_bytes(PASS, MODE);
+  unsigned char* region = smem + warp_id() * kRegion;
   uint32_t* rk = reinterpret_cast<uint32_t*>(region);
-  V* rv = reinterpret_cast<V*>(region + (PASS == 0 ? 0u : wr_num_val_offset<V>()));
-  const uint32_t cap = PASS == 0 ? wr_sym_cap() : wr_num_cap<V>();
+  V* rv = reinterpret_cast<V*>(region + (PASS == 0 ? 0u : wr_num_val_offset<V>(kRegion)));
+  const uint32_t cap = PASS == 0 ? wr_sym_cap() : wr_num_cap<V>(kRegion);
   const int64_t n = p.n_entries;
   constexpr bool kRange = PASS == 1 && MODE != 1;
   // row metadata, one field per lane: 0 A_rp[r], 1 A_rp[r+1], 2 prods[r] / C_rp[r], 3 C_rp[r+1],
