@@ -120,7 +120,8 @@ constexpr int kWarpRowCtasPerSMSym = 6;
 static_assert((kWarpRegionBytesSym * (kWarpRowThreads / 32) + 1024) * kWarpRowCtasPerSMSym <= kSmemPerSM, "warp-row CTAs");
 // numeric tiny rows (<= kTinyCnt entries, MODE 1): 2 KB regions hold 2.5x 64 entries, so the
 // smem no longer caps the CTAs; 5 CTAs (40 warps, 48 registers) measured best (C2 numeric A*P
-// 2.64 -> 2.56 ms; 6 CTAs at 40 registers spill and lose: 2.61 ms; ty_* runs, round 1)
+// 2.64 -> 2.56 ms; 6 CTAs at 40 registers spill and lose: 2.61 ms; ty_* runs, round 1), and
+// 2 products per lane per chunk instead of 4 at the same geometry: 2.56 -> 2.35 ms
 constexpr int kWarpRegionBytesTiny = 2048;
 constexpr int kWarpRowCtasPerSMTiny = 5;
 static_assert((kWarpRegionBytesTiny * (kWarpRowThreads / 32) + 1024) * kWarpRowCtasPerSMTiny <= kSmemPerSM, "warp-row CTAs");

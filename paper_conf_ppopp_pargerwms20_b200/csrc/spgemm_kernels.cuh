@@ -765,9 +765,9 @@ __device__ __forceinline__ int warp_row(const SpgemmArgs<V>& p, uint32_t* rk, V*
   // short rows keep the scrambled hash (robust to clustered columns) and rank counting
   const bool ordered = PASS == 1 && (MODE == 2 || (MODE == 0 && cnt > kSmallSeg));
   int newc = 0, wrapped = 0;
-  // numeric rows of the ordered map: 2 products per lane per chunk (fewer registers; C5 numeric
-  // 379 -> 362 ms), symbolic and tiny rows 4 (more loads in flight)
-  expand_row<PASS, V, PASS == 0, false, (PASS == 1 && MODE == 2) ? 2 : kPPL>(
+  // numeric MODE 1/2 rows: 2 products per lane per chunk (fewer registers; C5 numeric 379 -> 362 ms,
+  // C2 tiny rows at 40 warps/SM 2.56 -> 2.35 ms), symbolic and MODE 0 rows 4 (more loads in flight)
+  expand_row<PASS, V, PASS == 0, false, (PASS == 1 && MODE >= 1) ? 2 : kPPL>(
       p, a0, alen, 0, 1, [&](uint32_t col, V v, bool act) {
     if (PASS == 0) {
       if (act) newc += hash_insert_key(rk, S, col);
