@@ -765,9 +765,10 @@ __device__ __forceinline__ int warp_row(const SpgemmArgs<V>& p, uint32_t* rk, V*
   // short rows keep the scrambled hash (robust to clustered columns) and rank counting
   const bool ordered = PASS == 1 && (MODE == 2 || (MODE == 0 && cnt > kSmallSeg));
   int newc = 0, wrapped = 0;
-  // numeric MODE 1/2 rows: 2 products per lane per chunk (fewer registers; C5 numeric 379 -> 362 ms,
-  // C2 tiny rows at 40 warps/SM 2.56 -> 2.35 ms), symbolic and MODE 0 rows 4 (more loads in flight)
-  expand_row<PASS, V, PASS == 0, false, (PASS == 1 && MODE >= 1) ? 2 : kPPL>(
+  // 2 products per lane per chunk (fewer registers, more resident warps) for numeric MODE 1/2 rows
+  // (C5 numeric 379 -> 362 ms, C2 tiny rows at 40 warps/SM 2.56 -> 2.35 ms) and symbolic rows
+  // (C2 symbolic A*P 1.38 -> 1.31 ms; 8 per lane spills: 1.72 ms); numeric MODE 0 rows 4
+  expand_row<PASS, V, PASS == 0, false, (PASS == 0 || MODE >= 1) ? 2 : kPPL>(
       p, a0, alen, 0, 1, [&](uint32_t col, V v, bool act) {
     if (PASS == 0) {
       if (act) newc += hash_insert_key(rk, S, col);
