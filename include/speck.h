@@ -89,9 +89,59 @@ typedef enum {
   SPECK_OPT_SEGMENTS = 9,           /* 1: split rows beyond the largest map into column segments; 0: windowed dense [1] */
   SPECK_OPT_WARP_ROWS = 10,         /* 1: smallest bin = one warp per row (k_warp_rows); 0: merged blocks (Alg. 2) [1] */
   SPECK_OPT_LONG_BITMAP = 11,       /* 1: many long rows -> one bitmap+rank CTA per row when the column range fits; 2: always [1] */
-  SPECK_OPT_BITMAP_REUSE = 12       /* 1: the symbolic step keeps the dense bitmaps of numeric long rows (workspace
+  SPECK_OPT_BITMAP_REUSE = 12,      /* 1: the symbolic step keeps the dense bitmaps of numeric long rows (workspace
                                        <= 1/4 of free memory) so the numeric step does not rebuild them [1] */
+  SPECK_OPT_KERNEL_TIMING = 13,     /* 1: time every kernel launch with CUDA events on the stream it runs on; read
+                                       by speck_get_stats (kernel_id / kernel_bin / kernel_ms) [0] */
+  SPECK_OPT_PATH_COUNTERS = 14,     /* 1: count the rows each accumulator path processes (path_rows); costs a few
+                                       atomics per row — tests and diagnostics only [0] */
+  SPECK_OPT_BUCKET_SORT = 15        /* rows whose products are mostly distinct columns use a counting sort on
+                                       column buckets instead of the hash map: 0 off, 1 numeric rows, 2 numeric
+                                       and symbolic rows [2] */
 } speck_option_t;
+/* Changing any option except STAGE_TIMING, CONCURRENT_STREAMS, GLOBAL_LB_NUMERIC, VALIDATE,
+ * KERNEL_TIMING and PATH_COUNTERS after speck_analyze invalidates the analysis: the next
+ * speck_spgemm returns SPECK_ERR_NOT_ANALYZED until speck_analyze runs again. */
+
+/* Kernel identities reported by SPECK_OPT_KERNEL_TIMING: id = kind * 16 + configuration. */
+typedef enum {
+  SPECK_KERNEL_ANALYSIS = 1,     /* row analysis (Alg. 1) */
+  SPECK_KERNEL_BINNING = 2,      /* classification + bin scatter (global load balancer) */
+  SPECK_KERNEL_SCAN = 3,         /* prefix sum of the C row sizes */
+  SPECK_KERNEL_SYM_WARP = 4,     /* symbolic, one warp per row (smallest bin) */
+  SPECK_KERNEL_SYM_BLOCK = 5,    /* symbolic, one CTA per row or merged block (+ configuration 0..4) */
+  SPECK_KERNEL_NUM_TINY = 6,     /* numeric rows of <= 64 entries, one warp per row (rank counting) */
+  SPECK_KERNEL_NUM_WARP = 7,     /* numeric, one warp per row (ordered map) */
+  SPECK_KERNEL_NUM_BLOCK = 8,    /* numeric, one CTA per row or merged block (+ configuration 0..4) */
+  SPECK_KERNEL_DIRECT = 9,       /* numeric single-NZ rows (direct referencing) */
+  SPECK_KERNEL_SEGMENTS = 10,    /* numeric long rows: column segments / windows */
+  SPECK_KERNEL_LONG_BITMAP = 11, /* numeric long rows: bitmap + rank CTAs */
+  SPECK_KERNEL_SEG_PLAN = 12     /* long-row job planning */
+} speck_kernel_kind_t;
+
+/* Accumulator paths counted by SPECK_OPT_PATH_COUNTERS (rows per path, path_rows[]). */
+typedef enum {
+  SPECK_PATH_SYM_WARP = 0,        /* symbolic warp-per-row hash */
+  SPECK_PATH_SYM_BLOCK_HASH = 1,  /* symbolic hash shared by the warps of a CTA */
+  SPECK_PATH_SYM_MERGED = 2,      /* symbolic merged block (Alg. 2), warp per row */
+  SPECK_PATH_SYM_DENSE = 3,       /* symbolic dense bitmap, one window */
+  SPECK_PATH_SYM_DENSE_MULTI = 4, /* symbolic dense bitmap, several windows (resume positions) */
+  SPECK_PATH_NUM_TINY = 5,        /* numeric scrambled hash + rank counting (<= 64 entries) */
+  SPECK_PATH_NUM_WARP_ORDERED = 6,/* numeric warp-per-row ordered map */
+  SPECK_PATH_NUM_WARP_SORTED = 7, /* numeric warp-per-row compaction + sort (scrambled / wrapped map) */
+  SPECK_PATH_NUM_BLOCK_ORDERED = 8,/* numeric CTA ordered map */
+  SPECK_PATH_NUM_BLOCK_SORTED = 9,/* numeric CTA compaction + sort */
+  SPECK_PATH_NUM_MERGED = 10,     /* numeric merged block (Alg. 2), warp per row */
+  SPECK_PATH_NUM_DENSE = 11,      /* numeric dense window, one window */
+  SPECK_PATH_NUM_DENSE_MULTI = 12,/* numeric dense, several windows */
+  SPECK_PATH_NUM_DIRECT = 13,     /* numeric direct referencing */
+  SPECK_PATH_SEG_HASH = 14,       /* long row column segment, ordered hash (per segment) */
+  SPECK_PATH_SEG_DENSE = 15,      /* long row column segment, dense (per segment) */
+  SPECK_PATH_SEG_WINDOWS = 16,    /* long row, sequential dense windows (per job) */
+  SPECK_PATH_LONG_BITMAP = 17,    /* long row, bitmap + rank CTA */
+  SPECK_PATH_LONG_BITMAP_SPLIT = 18,/* long row, bitmap kept by the symbolic step, split over CTAs (per CTA) */
+  SPECK_PATH_COUNT = 24
+} speck_path_t;
 
 /* Statistics of the last analyze/spgemm pair (speck_get_stats). */
 typedef struct {
@@ -109,6 +159,24 @@ typedef struct {
   int64_t workspace_bytes;       /* workspace currently held by the handle */
   int64_t kernel_launches;       /* kernels this handle has launched since speck_create (cumulative) */
   float ms_analysis, ms_symbolic_lb, ms_symbolic, ms_scan, ms_numeric_lb, ms_numeric; /* SPECK_OPT_STAGE_TIMING */
+  /* Per bin of the last analyze/spgemm: [pass 0 symbolic / 1 numeric][category], categories
+   * 0 empty, 1 direct, 2..6 configurations 0..4, 7 long (numeric), 8 tiny (numeric <= 64
+   * entries), 9 unused.  Rows, Σ nnz(A_i), Σ products and (numeric) Σ nnz(C_i) of the rows in
+   * the bin — the per-kernel algorithmic byte model of bench.py is built from them. */
+  int64_t bin_rows[2][10];
+  int64_t bin_nnza[2][10];
+  int64_t bin_products[2][10];
+  int64_t bin_nnzc[10];
+  /* SPECK_OPT_KERNEL_TIMING: the launches of the last analyze/spgemm pair in issue order:
+   * kernel id (speck_kernel_kind_t * 16 + configuration), the bin it processed (pass * 16 +
+   * category; -1: all rows / not a bin) and its CUDA-event time on its own stream (ms). */
+  int32_t n_kernels;
+  int32_t kernel_id[64];
+  int32_t kernel_bin[64];
+  float kernel_ms[64];
+  /* SPECK_OPT_PATH_COUNTERS: rows (or segments / CTAs, see speck_path_t) per path since the
+   * option was set (cumulative over calls). */
+  int64_t path_rows[SPECK_PATH_COUNT];
 } speck_stats_t;
 
 /* Create a handle on `device` (CUDA ordinal). */

@@ -178,28 +178,39 @@ def compare(rp_gpu, col_gpu, val_gpu, rp_ref, col_ref, val_ref, scale_ref, tol: 
     """north_star parity rule on one row block.
 
     row_ptr and col must be bit-exact; |c - r| <= tol·s per entry, and c == ±0 when s == 0.
-    Returns dict(ok, rp_ok, col_mismatch, first_bad, max_rel, n_viol).
+    A non-finite GPU value (NaN, ±Inf) always fails: inputs are finite by contract (reading
+    R14), so every reference value and scale is finite.  The test is written as
+    `not (rel <= tol)` so that a NaN anywhere in the arithmetic counts as a violation.
+    Returns dict(ok, rp_ok, col_mismatch, first_bad, max_rel, n_viol, n_nonfinite).
     """
     rp_gpu = np.asarray(rp_gpu, np.int64); rp_ref = np.asarray(rp_ref, np.int64)
-    rp_ok = rp_gpu.shape == rp_ref.shape and bool(np.array_equal(rp_gpu - rp_gpu[0], rp_ref - rp_ref[0]))
-    out = {"rp_ok": rp_ok, "col_mismatch": None, "first_bad": None, "max_rel": 0.0, "n_viol": 0}
+    rp_ok = rp_gpu.shape == rp_ref.shape and rp_gpu.size > 0 and \
+        bool(np.array_equal(rp_gpu - rp_gpu[0], rp_ref - rp_ref[0]))
+    out = {"rp_ok": rp_ok, "col_mismatch": None, "first_bad": None, "max_rel": 0.0, "n_viol": 0, "n_nonfinite": 0}
     if not rp_ok:
         out["ok"] = False
         return out
+    n = int(rp_ref[-1] - rp_ref[0])
     col_gpu = np.asarray(col_gpu); col_ref = np.asarray(col_ref)
+    c = np.asarray(val_gpu, np.float64); r = np.asarray(val_ref, np.float64); s = np.asarray(scale_ref, np.float64)
+    if not (col_gpu.size == col_ref.size == c.size == r.size == s.size == n):
+        out["ok"] = False
+        out["col_mismatch"] = -1           # array lengths disagree with row_ptr
+        return out
     neq = np.nonzero(col_gpu != col_ref)[0]
     out["col_mismatch"] = int(neq.size)
     if neq.size:
         out["first_bad"] = int(neq[0])
         out["ok"] = False
         return out
-    c = np.asarray(val_gpu, np.float64); r = np.asarray(val_ref, np.float64); s = np.asarray(scale_ref, np.float64)
     err = np.abs(c - r)
     with np.errstate(divide="ignore", invalid="ignore"):
-        rel = np.where(s > 0, err / np.where(s > 0, s, 1.0), np.where(err > 0, np.inf, 0.0))
-    bad = rel > tol
+        rel = np.where(s > 0, err / np.where(s > 0, s, 1.0), np.where(err == 0, 0.0, np.inf))
+    nonfinite = ~np.isfinite(c)
+    bad = ~(rel <= tol) | nonfinite
+    out["n_nonfinite"] = int(nonfinite.sum())
     out["n_viol"] = int(bad.sum())
-    out["max_rel"] = float(rel.max()) if rel.size else 0.0
+    out["max_rel"] = float(np.max(np.where(np.isnan(rel), np.inf, rel))) if rel.size else 0.0
     if out["n_viol"]:
         out["first_bad"] = int(np.nonzero(bad)[0][0])
     out["ok"] = out["n_viol"] == 0

@@ -204,21 +204,46 @@ __global__ void __launch_bounds__(256) k_analysis_long(const int64_t* __restrict
 // ------------------------------------------------------------------------------------
 __global__ void __launch_bounds__(kBinTile) k_classify(const int64_t* __restrict__ A_rp, const int64_t* __restrict__ prods,
                                                        const int64_t* __restrict__ C_rp, int64_t m, BinParams bp,
-                                                       int64_t* __restrict__ hist, int64_t n_tiles) {
+                                                       int64_t* __restrict__ hist, int64_t n_tiles,
+                                                       unsigned long long* __restrict__ bin_sums) {
+  // per category: rows (histogram) and, for the statistics / per-kernel byte model, the sums
+  // of nnz(A_i), products and (numeric) nnz(C_i) — bin_sums[cat * 3 + {0, 1, 2}]
   __shared__ int cnt[CAT_COUNT];
+  __shared__ unsigned long long sums[CAT_COUNT][3];
   if (threadIdx.x < CAT_COUNT) cnt[threadIdx.x] = 0;
+  if (threadIdx.x < CAT_COUNT * 3) sums[threadIdx.x / 3][threadIdx.x % 3] = 0ull;
   __syncthreads();
   const int64_t row = (int64_t)blockIdx.x * kBinTile + threadIdx.x;
   if (row < m) {
     const int64_t nnza = A_rp[row + 1] - A_rp[row];
     const int64_t c = bp.pass ? C_rp[row + 1] - C_rp[row] : 0;
-    const int cat = classify_row(nnza, prods[row], c, bp);
+    const int64_t p = prods[row];
+    const int cat = classify_row(nnza, p, c, bp);
     // warp-aggregated increment
     const uint32_t peers = __match_any_sync(__activemask(), cat);
     if (lane_id() == __ffs(peers) - 1) atomicAdd(&cnt[cat], __popc(peers));
+    if (bin_sums) {
+      // warp-aggregated: sum over the lanes of the same category in 16-bit halves (rows < 2^40)
+      auto wsum = [&](unsigned long long x) {
+        const unsigned lo = __reduce_add_sync(peers, (unsigned)(x & 0xffffu));
+        const unsigned hi = __reduce_add_sync(peers, (unsigned)(x >> 16));
+        return (unsigned long long)lo + ((unsigned long long)hi << 16);
+      };
+      const unsigned long long s0 = wsum((unsigned long long)nnza), s1 = wsum((unsigned long long)p),
+                               s2 = bp.pass ? wsum((unsigned long long)c) : 0ull;
+      if (lane_id() == __ffs(peers) - 1) {
+        atomicAdd(&sums[cat][0], s0);
+        atomicAdd(&sums[cat][1], s1);
+        if (bp.pass) atomicAdd(&sums[cat][2], s2);
+      }
+    }
   }
   __syncthreads();
   if (threadIdx.x < CAT_COUNT) hist[(int64_t)threadIdx.x * n_tiles + blockIdx.x] = cnt[threadIdx.x];
+  if (bin_sums && threadIdx.x < CAT_COUNT * 3) {
+    const unsigned long long v = sums[threadIdx.x / 3][threadIdx.x % 3];
+    if (v) atomicAdd(&bin_sums[threadIdx.x], v);
+  }
 }
 
 // ------------------------------------------------------------------------------------

@@ -254,7 +254,8 @@ __global__ void __launch_bounds__(kCfgThreads[kSegCfg], 1024 / kCfgThreads[kSegC
 // Long rows by bitmap + rank (B200 design for rows beyond the largest hash map whose column
 // range fits a shared-memory bitmap; C3's ~175k long rows): one CTA of 1024 threads per row.
 //   1. structure: every product sets its column's bit (the symbolic pass's dense bitmap,
-//      P:1064-1084, recomputed: nothing survives between analyze and spgemm);
+//      P:1064-1084) — or, when the symbolic step kept this row's bitmap in the pool
+//      (SPECK_OPT_BITMAP_REUSE), the bitmap is loaded from there and no product is expanded;
 //   2. one block scan gives every 32-bit word its exclusive prefix = the output position of
 //      its first entry; C.col is written in order from the bitmap (sorted by construction)
 //      and the row's C.val range is zeroed;

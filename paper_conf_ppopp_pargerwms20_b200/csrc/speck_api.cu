@@ -31,6 +31,14 @@ struct Buf {
   size_t cap = 0;
 };
 
+constexpr int kMaxTimed = 64;      // timed launches per analyze/spgemm pair (SPECK_OPT_KERNEL_TIMING)
+constexpr int kPinnedWords = 256;  // pinned readback words
+// pinned readback layout (u64 words)
+constexpr int kPinSymCat = 16;     // [CAT_COUNT + 1] bin offsets
+constexpr int kPinBinSums = 64;    // [2][CAT_COUNT][3] per-bin sums (nnzA, products, nnzC)
+// `small` device scratch layout (bytes)
+constexpr int kSmallBinSums = 3072;   // unsigned long long [2][CAT_COUNT][3]
+
 }  // namespace speck
 
 using namespace speck;
@@ -38,13 +46,14 @@ using namespace speck;
 struct speck_handle_s {
   int device = 0;
   int num_sms = 148;
+  int num_smid = 148;   // %nsmid: bound of %smid (sizes the per-SM resume scratch)
   std::string err;
   // options
   int64_t opt_lb_sym = -1, opt_lb_num = -1, opt_force_acc = 0, opt_dense_window = 0, opt_timing = 0, opt_validate = 0,
-          opt_disable_direct = 0, opt_fixed_g = 0, opt_streams = 4;
+          opt_disable_direct = 0, opt_fixed_g = 0, opt_streams = 4, opt_esc = 2;
   // workspace
   Buf prods, maxlen, colmin, colmax, cnt, hist, hist_off, bins, stats, scan_status, resume, small, ana_long, binfo;
-  unsigned long long* h_pinned = nullptr;  // pinned readback area (64 x u64)
+  unsigned long long* h_pinned = nullptr;  // pinned readback area (kPinnedWords x u64)
   cudaStream_t streams[kMaxStreams] = {};
   cudaEvent_t ev_fork = nullptr, ev_join[kMaxStreams] = {};
   cudaEvent_t ev_t[8] = {};
@@ -71,6 +80,14 @@ struct speck_handle_s {
   int seg_shift = 15, nchunks = 0;
   int64_t long_thr = INT64_MAX, n_cand = 0, n_segs = 0, cand_start = 0;
   Buf chunk_cnt, cand, nseg, seg_off, segs;
+  // SPECK_OPT_KERNEL_TIMING: one event pair per launch of the current analyze/spgemm pair
+  int64_t opt_ktime = 0, opt_paths = 0;
+  cudaEvent_t kt_ev[2 * kMaxTimed] = {};
+  int kt_n = 0;
+  int32_t kt_id[kMaxTimed] = {}, kt_bin[kMaxTimed] = {};
+  float kt_ms[kMaxTimed] = {};
+  bool kt_pending = false;
+  Buf paths;   // SPECK_OPT_PATH_COUNTERS: unsigned long long [SPECK_PATH_COUNT]
   // user workspace allocator (speck_set_allocator)
   speck_alloc_fn ualloc = nullptr;
   speck_release_fn urelease = nullptr;
@@ -137,6 +154,20 @@ speck_status_t ensure(speck_handle_t h, Buf& b, size_t bytes, cudaStream_t s, bo
   return SPECK_OK;
 }
 
+// SPECK_OPT_KERNEL_TIMING: bracket a launch with events on the stream it runs on.
+int kt_begin(speck_handle_t h, cudaStream_t s, int kind, int cfg, int bin) {
+  if (!h->opt_ktime || h->kt_n >= kMaxTimed) return -1;
+  const int i = h->kt_n++;
+  h->kt_id[i] = kind * 16 + cfg;
+  h->kt_bin[i] = bin;
+  cudaEventRecord(h->kt_ev[2 * i], s);
+  h->kt_pending = true;
+  return i;
+}
+void kt_end(speck_handle_t h, cudaStream_t s, int i) {
+  if (i >= 0) cudaEventRecord(h->kt_ev[2 * i + 1], s);
+}
+
 int64_t ws_bytes(speck_handle_t h) {
   return (int64_t)(h->prods.cap + h->maxlen.cap + h->colmin.cap + h->colmax.cap + h->cnt.cap + h->hist.cap +
                    h->hist_off.cap + h->bins.cap + h->stats.cap + h->scan_status.cap + h->resume.cap + h->small.cap +
@@ -173,6 +204,7 @@ speck_status_t run_analysis(speck_handle_t h, const speck_csr_t* A, const speck_
   unsigned* nlong = reinterpret_cast<unsigned*>(static_cast<char*>(h->small.p) + 640);
   int32_t* lrows = static_cast<int32_t*>(h->ana_long.p);
   CK(cudaMemsetAsync(nlong, 0, 4, s));
+  const int kt = kt_begin(h, s, SPECK_KERNEL_ANALYSIS, 0, -1);
   // rows of B referenced several times on average: one 16-byte record per row of B
   const int4* binfo = nullptr;
   if (B->rows > 0 && A->nnz > 4 * B->rows && B->rows < ((int64_t)1 << 31)) {
@@ -200,6 +232,7 @@ speck_status_t run_analysis(speck_handle_t h, const speck_csr_t* A, const speck_
   k_analysis_long<<<(unsigned)h->num_sms * 2, 256, 0, s>>>(A->row_ptr, A->col_idx, B->row_ptr, B->col_idx, prods, maxlen,
                                                            colmin, colmax, st, lrows, nlong);
   CKL();
+  kt_end(h, s, kt);
   return SPECK_OK;
 }
 
@@ -221,12 +254,14 @@ void* spgemm_fn(int cfg, int pass) {
 }
 
 template <typename V>
-speck_status_t launch_spgemm(speck_handle_t h, int cfg, int pass, const SpgemmArgs<V>& a, cudaStream_t s) {
+speck_status_t launch_spgemm(speck_handle_t h, int cfg, int pass, const SpgemmArgs<V>& a, cudaStream_t s, int bin) {
   if (a.n_entries <= 0) return SPECK_OK;
   const int64_t grid = (a.n_entries + a.group_rows - 1) / a.group_rows;
   void* fn = spgemm_fn<V>(cfg, pass);
   void* args[] = {(void*)&a};
+  const int kt = kt_begin(h, s, pass == 0 ? SPECK_KERNEL_SYM_BLOCK : SPECK_KERNEL_NUM_BLOCK, cfg, bin);
   CK(cudaLaunchKernel(fn, dim3((unsigned)grid), dim3(kCfgThreads[cfg]), args, (size_t)kCfgMapBytes[cfg], s));
+  kt_end(h, s, kt);
   ++h->launches;
   return SPECK_OK;
 }
@@ -280,7 +315,7 @@ int64_t warp_row_fill(speck_handle_t h, int pass) {
 // Small-row kernel: persistent CTAs of 8 warps pulling rows from a counter (zeroed here).
 // mode (numeric): 0 any row, 1 rows of <= kTinyCnt entries, 2 larger rows (k_warp_rows MODE).
 template <typename V>
-speck_status_t launch_warp_rows(speck_handle_t h, int pass, const SpgemmArgs<V>& a, cudaStream_t s, int mode = 0) {
+speck_status_t launch_warp_rows(speck_handle_t h, int pass, const SpgemmArgs<V>& a, cudaStream_t s, int mode, int bin) {
   if (a.n_entries <= 0) return SPECK_OK;
   unsigned long long* ctr =
       reinterpret_cast<unsigned long long*>(static_cast<char*>(h->small.p) + 1024 + 8 * (pass == 0 ? 0 : 1 + mode));
@@ -288,11 +323,14 @@ speck_status_t launch_warp_rows(speck_handle_t h, int pass, const SpgemmArgs<V>&
   const int md = pass == 0 ? 0 : mode;
   const int64_t grid = std::min<int64_t>((a.n_entries + 7) / 8, (int64_t)h->num_sms * wr_ctas_per_sm(pass, md));
   const size_t smem = (size_t)wr_region_bytes(pass, md) * (kWarpRowThreads / 32);
+  const int kt = kt_begin(h, s, pass == 0 ? SPECK_KERNEL_SYM_WARP : md == 1 ? SPECK_KERNEL_NUM_TINY : SPECK_KERNEL_NUM_WARP,
+                          md, bin);
   if (pass == 0) k_warp_rows<0, V, 0><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
   else if (mode == 1) k_warp_rows<1, V, 1><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
   else if (mode == 2) k_warp_rows<1, V, 2><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
   else k_warp_rows<1, V, 0><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
   CKL();
+  kt_end(h, s, kt);
   return SPECK_OK;
 }
 
@@ -363,9 +401,11 @@ SpgemmArgs<V> base_args(speck_handle_t h, const speck_csr_t* A, const speck_csr_
   a.force_acc = (int)h->opt_force_acc;
   a.dense_window_cap = h->opt_dense_window;
   a.fixed_g = (int)h->opt_fixed_g;
+  a.esc = (int)h->opt_esc;
   a.cnt = static_cast<int64_t*>(h->cnt.p);
   a.resume = static_cast<int32_t*>(h->resume.p);
   a.resume_stride = 2 * std::max<int64_t>(h->max_nnza, 1);   // two buffers (cur / next) per SM slot
+  a.resume_slots = h->num_smid;
   a.n_dense_rows = reinterpret_cast<unsigned long long*>(static_cast<char*>(h->small.p) + 256);
   return a;
 }
@@ -416,7 +456,7 @@ speck_status_t run_pass(speck_handle_t h, int pass, int lb, const int64_t* cat_s
     a.rows = nullptr;
     a.n_entries = m;
     if (h->opt_warp_rows && need_max <= warp_row_fill(h, pass))
-      return launch_warp_rows<V>(h, pass, a, s, pass == 1 && need_max <= kTinyCnt ? 1 : 0);
+      return launch_warp_rows<V>(h, pass, a, s, pass == 1 && need_max <= kTinyCnt ? 1 : 0, -1);
     int cfg = -1, R = 1;
     for (int c = 0; c < kNumCfg; ++c)
       if (need_max * kMaxGroupRows <= own.cap[c]) { cfg = c; R = kMaxGroupRows; break; }
@@ -429,7 +469,7 @@ speck_status_t run_pass(speck_handle_t h, int pass, int lb, const int64_t* cat_s
     a.n_entries = m;
     a.group_rows = R;
     a.merge = 0;
-    return launch_spgemm<V>(h, cfg, pass, a, s);
+    return launch_spgemm<V>(h, cfg, pass, a, s, -1);
   }
   const int ns = (int)std::max<int64_t>(1, std::min<int64_t>(h->opt_streams, kMaxStreams));
   speck_status_t st;
@@ -438,10 +478,12 @@ speck_status_t run_pass(speck_handle_t h, int pass, int lb, const int64_t* cat_s
     // segment descriptors of the long rows (offsets were scanned during analyze)
     if ((st = ensure(h, h->segs, (size_t)h->n_segs * sizeof(Seg), s))) return st;
     const int64_t nc = h->n_cand;
+    const int kt = kt_begin(h, s, SPECK_KERNEL_SEG_PLAN, 1, -1);
     k_seg_emit<<<(unsigned)((nc + 127) / 128), 128, 0, s>>>(seg_plan_args<V>(h, a.C_rp),
                                                            static_cast<const int64_t*>(h->seg_off.p),
                                                            static_cast<Seg*>(h->segs.p));
     CKL();
+    kt_end(h, s, kt);
   }
   // few long rows with kept bitmaps: split them over several CTAs (zero C.val first, on the
   // user stream, before any kernel of this pass writes it)
@@ -459,15 +501,19 @@ speck_status_t run_pass(speck_handle_t h, int pass, int lb, const int64_t* cat_s
   if (pass == 1 && h->seg_enabled && h->n_cand > 0) {
     const SegPlanArgs sa = sa0;
     if (sa.bitmap_cols > 0) {
+      const int kt = kt_begin(h, h->streams[si], SPECK_KERNEL_LONG_BITMAP, 0, 16 + CAT_LONG);
       k_long_bitmap<V><<<(unsigned)(h->n_cand * sa.split_max), kBitmapThreads, kCfgMapBytes[kNumCfg - 1], h->streams[si]>>>(a, sa);
       CKL();
+      kt_end(h, h->streams[si], kt);
       si = (si + 1) % ns;
     }
   }
   if (segs) {
+    const int kt = kt_begin(h, h->streams[si], SPECK_KERNEL_SEGMENTS, kSegCfg, 16 + CAT_LONG);
     k_segments<V><<<(unsigned)h->n_segs, kCfgThreads[kSegCfg], kCfgMapBytes[kSegCfg], h->streams[si]>>>(
         a, static_cast<const Seg*>(h->segs.p));
     CKL();
+    kt_end(h, h->streams[si], kt);
     si = (si + 1) % ns;
   }
   // largest configurations first so long rows start early
@@ -479,7 +525,7 @@ speck_status_t run_pass(speck_handle_t h, int pass, int lb, const int64_t* cat_s
     b.rows = bins + cat_start[cat];
     b.n_entries = n;
     if (c == 0 && h->opt_warp_rows) {
-      st = launch_warp_rows<V>(h, pass, b, h->streams[si], pass == 1 ? 2 : 0);
+      st = launch_warp_rows<V>(h, pass, b, h->streams[si], pass == 1 ? 2 : 0, pass * 16 + cat);
       if (st) return st;
       si = (si + 1) % ns;
       continue;
@@ -504,7 +550,7 @@ speck_status_t run_pass(speck_handle_t h, int pass, int lb, const int64_t* cat_s
         b.bm_off = static_cast<int64_t*>(h->bm_off.p);
       }
     }
-    st = launch_spgemm<V>(h, c, pass, b, h->streams[si]);
+    st = launch_spgemm<V>(h, c, pass, b, h->streams[si], pass * 16 + cat);
     if (st) return st;
     si = (si + 1) % ns;
   }
@@ -512,7 +558,7 @@ speck_status_t run_pass(speck_handle_t h, int pass, int lb, const int64_t* cat_s
     SpgemmArgs<V> b = a;
     b.rows = bins + cat_start[CAT_TINY];
     b.n_entries = cat_start[CAT_TINY + 1] - cat_start[CAT_TINY];
-    st = launch_warp_rows<V>(h, pass, b, h->streams[si], 1);
+    st = launch_warp_rows<V>(h, pass, b, h->streams[si], 1, 16 + CAT_TINY);
     if (st) return st;
     si = (si + 1) % ns;
   }
@@ -526,6 +572,7 @@ speck_status_t run_pass(speck_handle_t h, int pass, int lb, const int64_t* cat_s
       const unsigned grid = (unsigned)std::min<int64_t>((n + rows_per_cta - 1) / rows_per_cta, (int64_t)h->num_sms * 16);
       const int32_t* rows = bins + cat_start[CAT_DIRECT];
       cudaStream_t ds = h->streams[si];
+      const int kt = kt_begin(h, ds, SPECK_KERNEL_DIRECT, 0, 16 + CAT_DIRECT);
 #define SPECK_DIRECT(GD)                                                                                   \
   k_direct<V, GD><<<grid, 256, 0, ds>>>(rows, n, a.A_rp, a.A_col, a.A_val, a.B_rp, a.B_col, a.B_val, a.C_rp, \
                                         a.C_col, a.C_val)
@@ -539,6 +586,7 @@ speck_status_t run_pass(speck_handle_t h, int pass, int lb, const int64_t* cat_s
       }
 #undef SPECK_DIRECT
       CKL();
+      kt_end(h, ds, kt);
     }
   }
   return join(h, s, ns);
@@ -567,7 +615,14 @@ speck_status_t analyze_impl(speck_handle_t h, const speck_csr_t* A, const speck_
   h->dtype = A->dtype;
   h->A_rp = A->row_ptr; h->A_col = A->col_idx; h->A_rows = A->rows; h->A_cols = A->cols; h->A_nnz = A->nnz;
   h->B_rp = B->row_ptr; h->B_col = B->col_idx; h->B_rows = B->rows; h->B_cols = B->cols; h->B_nnz = B->nnz;
-  std::memset(&h->st, 0, sizeof h->st);
+  {
+    int64_t keep[SPECK_PATH_COUNT];   // path counters are cumulative
+    std::memcpy(keep, h->st.path_rows, sizeof keep);
+    std::memset(&h->st, 0, sizeof h->st);
+    std::memcpy(h->st.path_rows, keep, sizeof keep);
+  }
+  h->kt_n = 0;
+  h->kt_pending = false;
   plan_segments<V>(h, B->cols);
   if (m == 0) {
     if (C_rp) CK(cudaMemsetAsync(C_rp, 0, sizeof(int64_t), s));
@@ -608,25 +663,34 @@ speck_status_t analyze_impl(speck_handle_t h, const speck_csr_t* A, const speck_
     return st;
   // symbolic classification histogram per tile (global LB step 1), computed unconditionally
   const BinParams bps = make_bin_params(h, 0);
+  unsigned long long* bin_sums = reinterpret_cast<unsigned long long*>(static_cast<char*>(h->small.p) + kSmallBinSums);
+  int kt = kt_begin(h, s, SPECK_KERNEL_BINNING, 0, -1);
   k_classify<<<(unsigned)tiles, kBinTile, 0, s>>>(A->row_ptr, static_cast<int64_t*>(h->prods.p), nullptr, m, bps,
-                                                 static_cast<int64_t*>(h->hist.p), tiles);
+                                                 static_cast<int64_t*>(h->hist.p), tiles, bin_sums);
   CKL();
   if ((st = launch_scan(h, static_cast<int64_t*>(h->hist.p), tiles * CAT_COUNT, static_cast<int64_t*>(h->hist_off.p),
                         nullptr, s)))
     return st;
+  kt_end(h, s, kt);
   // read back the stats and the bin boundaries (sync #1)
   {
     unsigned long long* hp = h->h_pinned;
     CK(cudaMemcpyAsync(hp, dstats, sizeof(AnalysisStats), cudaMemcpyDeviceToHost, s));
     for (int c = 0; c <= CAT_COUNT; ++c)
-      CK(cudaMemcpyAsync(hp + 16 + c, static_cast<int64_t*>(h->hist_off.p) + (int64_t)c * tiles, 8,
+      CK(cudaMemcpyAsync(hp + kPinSymCat + c, static_cast<int64_t*>(h->hist_off.p) + (int64_t)c * tiles, 8,
                          cudaMemcpyDeviceToHost, s));
+    CK(cudaMemcpyAsync(hp + kPinBinSums, bin_sums, CAT_COUNT * 3 * 8, cudaMemcpyDeviceToHost, s));
     CK(cudaStreamSynchronize(s));
   }
   AnalysisStats hs;
   std::memcpy(&hs, h->h_pinned, sizeof hs);
   int64_t sym_cat[CAT_COUNT + 1];
-  for (int c = 0; c <= CAT_COUNT; ++c) sym_cat[c] = (int64_t)h->h_pinned[16 + c];
+  for (int c = 0; c <= CAT_COUNT; ++c) sym_cat[c] = (int64_t)h->h_pinned[kPinSymCat + c];
+  for (int c = 0; c < CAT_COUNT; ++c) {
+    h->st.bin_rows[0][c] = sym_cat[c + 1] - sym_cat[c];
+    h->st.bin_nnza[0][c] = (int64_t)h->h_pinned[kPinBinSums + 3 * c];
+    h->st.bin_products[0][c] = (int64_t)h->h_pinned[kPinBinSums + 3 * c + 1];
+  }
   h->max_nnza = (int64_t)hs.max_nnza;
   h->st.products = (int64_t)hs.sum_prods;
   h->st.max_row_products = (int64_t)hs.max_prods;
@@ -636,7 +700,7 @@ speck_status_t analyze_impl(speck_handle_t h, const speck_csr_t* A, const speck_
   if ((st = timing_mark(h, 1, s))) return st;
 
   // resume scratch for multi-window dense rows (largest configuration, one CTA per SM)
-  if ((st = ensure(h, h->resume, (size_t)h->num_sms * 2 * (size_t)std::max<int64_t>(h->max_nnza, 1) * 4, s))) return st;
+  if ((st = ensure(h, h->resume, (size_t)h->num_smid * 2 * (size_t)std::max<int64_t>(h->max_nnza, 1) * 4, s))) return st;
 
   // ---- 2. symbolic global load balancing decision + binning --------------------------
   const int cfg_max_sym = cfg_for(bps, (int64_t)hs.max_prods);
@@ -683,10 +747,12 @@ speck_status_t analyze_impl(speck_handle_t h, const speck_csr_t* A, const speck_
   }
   SpgemmArgs<V> a = base_args<V>(h, A, B);
   if (lb_sym) {
+    kt = kt_begin(h, s, SPECK_KERNEL_BINNING, 1, -1);
     k_bin_scatter<<<(unsigned)tiles, kBinTile, 0, s>>>(A->row_ptr, static_cast<int64_t*>(h->prods.p), nullptr, m, bps,
                                                       static_cast<int64_t*>(h->hist_off.p), tiles,
                                                       static_cast<int32_t*>(h->bins.p), static_cast<int64_t*>(h->cnt.p));
     CKL();
+    kt_end(h, s, kt);
   }
   if ((st = timing_mark(h, 2, s))) return st;
   // ---- 3. symbolic SpGEMM -------------------------------------------------------------
@@ -694,15 +760,19 @@ speck_status_t analyze_impl(speck_handle_t h, const speck_csr_t* A, const speck_
   if ((st = timing_mark(h, 3, s))) return st;
   // ---- 4. prefix sum -> C row offsets; numeric classification -------------------------
   unsigned long long* dmax = reinterpret_cast<unsigned long long*>(static_cast<char*>(h->small.p) + 128);
+  kt = kt_begin(h, s, SPECK_KERNEL_SCAN, 0, -1);
   if ((st = launch_scan(h, static_cast<int64_t*>(h->cnt.p), m, C_rp, dmax, s))) return st;
+  kt_end(h, s, kt);
   if ((st = timing_mark(h, 4, s))) return st;
   const BinParams bpn = make_bin_params(h, 1);
+  kt = kt_begin(h, s, SPECK_KERNEL_BINNING, 2, -1);
   k_classify<<<(unsigned)tiles, kBinTile, 0, s>>>(A->row_ptr, static_cast<int64_t*>(h->prods.p), C_rp, m, bpn,
-                                                 static_cast<int64_t*>(h->hist.p), tiles);
+                                                 static_cast<int64_t*>(h->hist.p), tiles, bin_sums + CAT_COUNT * 3);
   CKL();
   if ((st = launch_scan(h, static_cast<int64_t*>(h->hist.p), tiles * CAT_COUNT, static_cast<int64_t*>(h->hist_off.p),
                         nullptr, s)))
     return st;
+  kt_end(h, s, kt);
   // numeric long rows: segments per candidate (exact sizes from the symbolic chunk counts)
   if (h->seg_enabled && h->n_cand > 0) {
     const int64_t nc = h->n_cand;
@@ -711,11 +781,13 @@ speck_status_t analyze_impl(speck_handle_t h, const speck_csr_t* A, const speck_
     if ((st = ensure(h, h->seg_off, (size_t)(nc + 1) * 8, s))) return st;
     CK(cudaMemcpyAsync(h->cand.p, static_cast<int32_t*>(h->bins.p) + h->cand_start, (size_t)nc * 4,
                        cudaMemcpyDeviceToDevice, s));
+    kt = kt_begin(h, s, SPECK_KERNEL_SEG_PLAN, 0, -1);
     k_seg_count<<<(unsigned)((nc + 127) / 128), 128, 0, s>>>(seg_plan_args<V>(h, C_rp),
                                                             static_cast<int64_t*>(h->nseg.p));
     CKL();
     if ((st = launch_scan(h, static_cast<int64_t*>(h->nseg.p), nc, static_cast<int64_t*>(h->seg_off.p), nullptr, s)))
       return st;
+    kt_end(h, s, kt);
   }
   {
     unsigned long long* hp = h->h_pinned;
@@ -725,15 +797,23 @@ speck_status_t analyze_impl(speck_handle_t h, const speck_csr_t* A, const speck_
     if (h->seg_enabled && h->n_cand > 0)
       CK(cudaMemcpyAsync(hp + 2, static_cast<int64_t*>(h->seg_off.p) + h->n_cand, 8, cudaMemcpyDeviceToHost, s));
     for (int c = 0; c <= CAT_COUNT; ++c)
-      CK(cudaMemcpyAsync(hp + 16 + c, static_cast<int64_t*>(h->hist_off.p) + (int64_t)c * tiles, 8,
+      CK(cudaMemcpyAsync(hp + kPinSymCat + c, static_cast<int64_t*>(h->hist_off.p) + (int64_t)c * tiles, 8,
                          cudaMemcpyDeviceToHost, s));
+    CK(cudaMemcpyAsync(hp + kPinBinSums + CAT_COUNT * 3, bin_sums + CAT_COUNT * 3, CAT_COUNT * 3 * 8,
+                       cudaMemcpyDeviceToHost, s));
     CK(cudaStreamSynchronize(s));  // sync #2
   }
   h->nnz_c = (int64_t)h->h_pinned[0];
   h->max_cnt = (int64_t)h->h_pinned[1];
   h->n_segs = (int64_t)h->h_pinned[2];
   h->st.segments = h->n_segs;
-  for (int c = 0; c <= CAT_COUNT; ++c) h->num_cat_start[c] = (int64_t)h->h_pinned[16 + c];
+  for (int c = 0; c <= CAT_COUNT; ++c) h->num_cat_start[c] = (int64_t)h->h_pinned[kPinSymCat + c];
+  for (int c = 0; c < CAT_COUNT; ++c) {
+    h->st.bin_rows[1][c] = h->num_cat_start[c + 1] - h->num_cat_start[c];
+    h->st.bin_nnza[1][c] = (int64_t)h->h_pinned[kPinBinSums + CAT_COUNT * 3 + 3 * c];
+    h->st.bin_products[1][c] = (int64_t)h->h_pinned[kPinBinSums + CAT_COUNT * 3 + 3 * c + 1];
+    h->st.bin_nnzc[c] = (int64_t)h->h_pinned[kPinBinSums + CAT_COUNT * 3 + 3 * c + 2];
+  }
   for (int c = 0; c < CAT_TINY; ++c) h->st.rows_per_bin_numeric[c] = h->num_cat_start[c + 1] - h->num_cat_start[c];
   // the stats keep one smallest-configuration count (tiny rows included)
   h->st.rows_per_bin_numeric[CAT_CFG0] += h->num_cat_start[CAT_TINY + 1] - h->num_cat_start[CAT_TINY];
@@ -766,10 +846,12 @@ speck_status_t spgemm_impl(speck_handle_t h, const speck_csr_t* A, const speck_c
   unsigned long long* ndense = reinterpret_cast<unsigned long long*>(static_cast<char*>(h->small.p) + 256);
   CK(cudaMemsetAsync(ndense, 0, 8, s));
   if (lb) {
+    const int kt = kt_begin(h, s, SPECK_KERNEL_BINNING, 3, -1);
     k_bin_scatter<<<(unsigned)tiles, kBinTile, 0, s>>>(A->row_ptr, static_cast<int64_t*>(h->prods.p), C_rp, m, bpn,
                                                       static_cast<int64_t*>(h->hist_off.p), tiles,
                                                       static_cast<int32_t*>(h->bins.p), nullptr);
     CKL();
+    kt_end(h, s, kt);
   }
   if ((st = timing_mark(h, 6, s))) return st;
   SpgemmArgs<V> a = base_args<V>(h, A, B);
@@ -801,6 +883,8 @@ __global__ void k_block_merge_groups(const int64_t* needs, int64_t n, int64_t ca
   if (l < ne) flags[g0 + l] = (st >> l) & 1u;
 }
 
+__global__ void k_query_nsmid(int* out) { *out = (int)nsmid(); }
+
 __global__ void k_group_size(int32_t T, const int64_t* nnzA, const int64_t* prods, const int64_t* maxlen, int64_t n,
                              int32_t* g) {
   const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -815,10 +899,11 @@ __global__ void k_hash_probe(const uint32_t* keys, const uint32_t* homes, int64_
   for (int i = threadIdx.x; i < size; i += blockDim.x) { sk[i] = kEmptyKey; sc[i] = 0; }
   __syncthreads();
   if (threadIdx.x == 0) {
-    // the pipeline's probe_insert with the home slot injected instead of hash_slot()
+    // the pipeline's probe_insert_mono (numeric maps of scrambled rows) with the home slot
+    // injected instead of hash_slot()
+    int wrapped = 0;
     for (int64_t i = 0; i < n; ++i) {
-      bool is_new;
-      const uint32_t s = probe_insert(sk, (uint32_t)size, homes[i] % (uint32_t)size, keys[i], &is_new);
+      const uint32_t s = probe_insert_mono(sk, (uint32_t)size, homes[i] % (uint32_t)size, keys[i], &wrapped);
       atomicAdd(&sc[s], 1u);
     }
   }
@@ -867,12 +952,25 @@ speck_status_t speck_create(speck_handle_t* out, int device) {
   cudaGetDevice(&prev);
   if (cudaSetDevice(device) != cudaSuccess) { delete h; return SPECK_ERR_CUDA; }
   cudaDeviceGetAttribute(&h->num_sms, cudaDevAttrMultiProcessorCount, device);
-  bool ok = cudaHostAlloc(&h->h_pinned, 64 * 8, cudaHostAllocDefault) == cudaSuccess;
+  bool ok = cudaHostAlloc(&h->h_pinned, kPinnedWords * 8, cudaHostAllocDefault) == cudaSuccess;
   for (int i = 0; i < kMaxStreams && ok; ++i) ok = cudaStreamCreateWithFlags(&h->streams[i], cudaStreamNonBlocking) == cudaSuccess;
   ok = ok && cudaEventCreateWithFlags(&h->ev_fork, cudaEventDisableTiming) == cudaSuccess;
   for (int i = 0; i < kMaxStreams && ok; ++i) ok = cudaEventCreateWithFlags(&h->ev_join[i], cudaEventDisableTiming) == cudaSuccess;
   for (int i = 0; i < 8 && ok; ++i) ok = cudaEventCreate(&h->ev_t[i]) == cudaSuccess;
+  for (int i = 0; i < 2 * kMaxTimed && ok; ++i) ok = cudaEventCreate(&h->kt_ev[i]) == cudaSuccess;
   if (ok) ok = set_smem_attrs<float>(h) == SPECK_OK && set_smem_attrs<double>(h) == SPECK_OK;
+  if (ok) {
+    // %nsmid bounds %smid (it may exceed the SM count): it sizes the per-SM resume slots
+    int* d = nullptr;
+    ok = cudaMalloc(&d, sizeof(int)) == cudaSuccess;
+    if (ok) {
+      k_query_nsmid<<<1, 1>>>(d);
+      int v = 0;
+      ok = cudaMemcpy(&v, d, sizeof(int), cudaMemcpyDeviceToHost) == cudaSuccess;
+      if (ok) h->num_smid = std::max(v, h->num_sms);
+      cudaFree(d);
+    }
+  }
   cudaSetDevice(prev);
   if (!ok) {
     (void)cudaGetLastError();
@@ -905,6 +1003,8 @@ speck_status_t speck_destroy(speck_handle_t h) {
   if (h->ev_fork) cudaEventDestroy(h->ev_fork);
   for (int i = 0; i < 8; ++i)
     if (h->ev_t[i]) cudaEventDestroy(h->ev_t[i]);
+  for (int i = 0; i < 2 * kMaxTimed; ++i)
+    if (h->kt_ev[i]) cudaEventDestroy(h->kt_ev[i]);
   (void)cudaGetLastError();
   cudaSetDevice(prev);
   delete h;
@@ -913,6 +1013,13 @@ speck_status_t speck_destroy(speck_handle_t h) {
 
 speck_status_t speck_set_option(speck_handle_t h, int option, int64_t v) {
   if (!h) return SPECK_ERR_INVALID_ARGUMENT;
+  // every option except these shapes the plan speck_analyze builds (bins, long-row jobs,
+  // bitmap pool): changing it invalidates the analysis, so a following speck_spgemm fails with
+  // SPECK_ERR_NOT_ANALYZED instead of running kernels on a stale plan
+  if (option != SPECK_OPT_STAGE_TIMING && option != SPECK_OPT_CONCURRENT_STREAMS &&
+      option != SPECK_OPT_GLOBAL_LB_NUMERIC && option != SPECK_OPT_VALIDATE && option != SPECK_OPT_KERNEL_TIMING &&
+      option != SPECK_OPT_PATH_COUNTERS)
+    h->analyzed = false;
   switch (option) {
     case SPECK_OPT_GLOBAL_LB_SYMBOLIC: h->opt_lb_sym = v; break;
     case SPECK_OPT_GLOBAL_LB_NUMERIC: h->opt_lb_num = v; break;
@@ -935,6 +1042,14 @@ speck_status_t speck_set_option(speck_handle_t h, int option, int64_t v) {
     case SPECK_OPT_WARP_ROWS: h->opt_warp_rows = v; break;
     case SPECK_OPT_LONG_BITMAP: h->opt_long_bitmap = v; break;
     case SPECK_OPT_BITMAP_REUSE: h->opt_bitmap_reuse = v; break;
+    case SPECK_OPT_KERNEL_TIMING: h->opt_ktime = v; break;
+    case SPECK_OPT_BUCKET_SORT:
+      if (v < 0 || v > 2) return fail(h, SPECK_ERR_INVALID_ARGUMENT, "BUCKET_SORT must be 0..2");
+      h->opt_esc = v; break;
+    case SPECK_OPT_PATH_COUNTERS:
+      h->opt_paths = v;
+      std::memset(h->st.path_rows, 0, sizeof h->st.path_rows);
+      break;
     default: return fail(h, SPECK_ERR_INVALID_ARGUMENT, "unknown option %d", option);
   }
   return SPECK_OK;
@@ -1041,6 +1156,24 @@ speck_status_t speck_get_stats(speck_handle_t h, speck_stats_t* out) {
     h->st.ms_numeric = elapsed(h, 6, 7);
     h->st.rows_dense_numeric = (int64_t)h->h_pinned[40];
     h->numeric_pending = false;
+  }
+  if (h->kt_pending) {
+    for (int i = 0; i < h->kt_n; ++i) {
+      float ms = -1.f;
+      if (cudaEventSynchronize(h->kt_ev[2 * i + 1]) != cudaSuccess ||
+          cudaEventElapsedTime(&ms, h->kt_ev[2 * i], h->kt_ev[2 * i + 1]) != cudaSuccess) {
+        (void)cudaGetLastError();
+        ms = -1.f;
+      }
+      h->kt_ms[i] = ms;
+    }
+    h->kt_pending = false;
+  }
+  h->st.n_kernels = h->kt_n;
+  for (int i = 0; i < h->kt_n; ++i) {
+    h->st.kernel_id[i] = h->kt_id[i];
+    h->st.kernel_bin[i] = h->kt_bin[i];
+    h->st.kernel_ms[i] = h->kt_ms[i];
   }
   h->st.workspace_bytes = ws_bytes(h);
   h->st.kernel_launches = h->launches;

@@ -172,8 +172,8 @@ __host__ __device__ inline int classify_row(int64_t nnza, int64_t prods, int64_t
   if (bp.use_direct && nnza == 1) return CAT_DIRECT;
   if (bp.pass == 1 && cnt > bp.long_thr) return CAT_LONG;
   int64_t need = bp.pass == 0 ? prods : cnt;
-#pragma unroll
   if (bp.pass == 1 && need <= bp.tiny_cap && need <= bp.cap[0]) return CAT_TINY;
+#pragma unroll
   for (int c = 0; c < kNumCfg - 1; ++c)
     if (need <= bp.cap[c]) return CAT_CFG0 + c;
   return CAT_CFG0 + kNumCfg - 1;
@@ -315,6 +315,7 @@ struct SpgemmArgs {
   int force_acc;             // 0 auto, 1 hash, 2 dense
   int64_t dense_window_cap;  // >0: cap dense window (test knob)
   int fixed_g;               // >0: fixed group size
+  int esc;                   // bucket counting-sort rows (esc_kernels.cuh): 0 off, 1 numeric, 2 + symbolic
   // symbolic out
   int64_t* cnt;
   // numeric in/out
@@ -324,6 +325,7 @@ struct SpgemmArgs {
   // resume-position scratch for multi-window dense rows: [num_sms][resume_stride]
   int32_t* resume;
   int64_t resume_stride;
+  int64_t resume_slots;      // slots in `resume` (%nsmid of the device)
   // counters
   unsigned long long* n_dense_rows;
   // symbolic, largest configuration: per-chunk counts of long-row candidates

@@ -23,6 +23,7 @@
 #pragma once
 
 #include "speck_internal.cuh"
+#include "esc_kernels.cuh"
 
 namespace speck {
 
@@ -43,7 +44,7 @@ struct BlockMeta {
   int32_t rhi[kMaxGroupRows];
   int32_t rwrap[kMaxGroupRows];      // block path: a probing run of the row wrapped around
   uint32_t starts;
-  int nr, g, dense, ordered;
+  int nr, g, dense, ordered, esc;
   int64_t nnzA, prods, maxlen, cnt;
   int32_t colmin, colmax;
   int64_t scan_part[33];
@@ -61,21 +62,6 @@ static_assert(cfg_fits<0>() && cfg_fits<1>() && cfg_fits<2>() && cfg_fits<3>() &
 
 template <typename V>
 __device__ __forceinline__ V ldv(const V* p) { return __ldg(p); }
-
-// Linear probing from slot s (Fig. 4): find `key` or claim an empty slot for
-// it with a CAS; returns the slot, *is_new tells whether this thread inserted the key.
-__device__ __forceinline__ uint32_t probe_insert(uint32_t* keys, uint32_t S, uint32_t s, uint32_t key, bool* is_new) {
-  while (true) {
-    const uint32_t k = keys[s];
-    if (k == key) { *is_new = false; return s; }
-    if (k == kEmptyKey) {
-      const uint32_t old = atomicCAS(&keys[s], kEmptyKey, key);
-      if (old == kEmptyKey) { *is_new = true; return s; }
-      if (old == key) { *is_new = false; return s; }
-    }
-    s = (s + 1 == S) ? 0u : s + 1;
-  }
-}
 
 // Order-preserving numeric maps: 8-slot buckets, the home bucket monotone in the column over
 // the row's [colmin, colmax] and covering the first 7/8 of the buckets (the rest absorbs
@@ -121,7 +107,11 @@ __device__ __forceinline__ uint32_t probe_insert_bkt(uint32_t* keys, uint32_t NB
   }
 }
 
-// linear probing that reports a wrap-around (which breaks the cluster order)
+// Linear probing from slot s (Fig. 4): find `key` or claim the first empty slot
+// with a CAS, moving to the next slot (mod S) while the slot holds another key; reports a
+// wrap-around past the last slot (which breaks the cluster order of monotone homes).  The
+// numeric maps of scrambled rows use it (home = hash_slot), and speck_hash_probe runs it with
+// injected homes for the Fig. 4 example.
 __device__ __forceinline__ uint32_t probe_insert_mono(uint32_t* keys, uint32_t S, uint32_t s, uint32_t key, int* wrapped) {
   while (true) {
     const uint32_t k = keys[s];
@@ -646,10 +636,19 @@ __device__ int64_t dense_emit(const uint32_t* bits, const V* dvals, int nwords, 
   return total;
 }
 
-// acquire a per-SM resume scratch slot (largest configuration: one CTA per SM)
+// Per-SM resume scratch slot of multi-window dense rows.  The slot is private because such
+// rows run only in the largest configuration, whose 225 KB of shared memory admits one CTA per
+// SM (no other kernel of any launch can co-reside with it: the bitmap kernel needs the same
+// 225 KB).  The buffer holds %nsmid slots (queried at speck_create; %smid < %nsmid, which may
+// exceed the SM count), and an out-of-range id traps instead of writing past the buffer.
 __device__ __forceinline__ unsigned smid() {
   unsigned r;
   asm volatile("mov.u32 %0, %%smid;" : "=r"(r));
+  return r;
+}
+__device__ __forceinline__ unsigned nsmid() {
+  unsigned r;
+  asm volatile("mov.u32 %0, %%nsmid;" : "=r"(r));
   return r;
 }
 
@@ -870,8 +869,8 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
       const int64_t need_tot = PASS == 0 ? tot_p : tot_c;
       uint32_t rsz = 0;
       // (multiples of 4 slots so 4-slot probe groups stay 16-byte aligned: 4 + a share of the rest)
-      // A single row gets a region sized to it (symbolic 1.5x products = 66% fill, numeric 2x
-      // entries = 50%), so clearing and the write-out scan touch only the slots the row can use
+      // A single row gets a region sized to it (symbolic 2x products, numeric 2.5x entries:
+      // <= 50% / 40% load), so clearing and the write-out scan touch only the slots the row can use
       // (C5: the write-out scan of the full map was over half of the numeric instructions).
       if (l < nr) {
         if (nr == 1) {
@@ -930,13 +929,41 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
           }
         }
         bm.dense = dense;
+        // single-row hash blocks whose products are (almost) all distinct: bucket counting sort
+        const int64_t ecap = esc_capacity<V>(PASS, kCfgMapBytes[CFG]);
+        bm.esc = (nr == 1 && !dense && tot_p > 0 && tot_p <= ecap && tot_p <= 32 * T &&
+                  p.esc >= (PASS == 0 ? 2 : 1) && (PASS == 0 || tot_p <= 2 * tot_c)) ? 1 : 0;
       }
     }
     __syncthreads();
     const int64_t nnzA = bm.nnzA;
     constexpr int NW = T / 32;
 
-    if (!bm.dense && nr >= NW && nr > 1) {
+    int esc_done = 0;
+    if (bm.esc) {
+      // ===================== BUCKET COUNTING SORT (esc_kernels.cuh) =====================
+      const bool chunks = CFG == kNumCfg - 1 && PASS == 0 && p.chunk_cnt && bm.prods > p.long_thr;
+      if (chunks) {
+        for (int i = tid; i < p.nchunks; i += T) chist[i] = 0;
+        __syncthreads();
+      }
+      const int c = esc_row<NW, PASS, V>(p, smem, kCfgMapBytes[CFG], warp_id(), bm.astart[0], (int)bm.nnzA,
+                                         (int)bm.prods, (int)bm.cnt, bm.colmin, bm.colmax, bm.cbase[0],
+                                         reinterpret_cast<int*>(bm.scan_part), chunks ? chist : nullptr,
+                                         p.chunk_shift);
+      if (c >= 0) {
+        esc_done = 1;
+        if (PASS == 0 && tid == 0) p.cnt[bm.row[b0]] = c;
+        if (chunks) {
+          __syncthreads();
+          int32_t* dst = p.chunk_cnt + (int64_t)blockIdx.x * p.nchunks;
+          for (int i = tid; i < p.nchunks; i += T) dst[i] = chist[i];
+        }
+      }
+      __syncthreads();
+    }
+    if (esc_done) {
+    } else if (!bm.dense && nr >= NW && nr > 1) {
       // ===================== HASH, WARP PER ROW (multi-row blocks) =====================
       // Each warp owns whole rows and their private map regions, so accumulation and the
       // sort/compaction epilogue need no block barrier; lanes whose key is unique within
@@ -1055,7 +1082,9 @@ __device__ __noinline__ void dense_row(const SpgemmArgs<V>& p, BlockMeta& bm, in
       int32_t* res = nullptr;       // double-buffered resume offsets (cur, next)
       int32_t* res_next = nullptr;
       if (nwin > 1) {
-        res = p.resume + (int64_t)smid() * p.resume_stride;
+        const unsigned slot = smid();
+        if (slot >= (unsigned)p.resume_slots) __trap();
+        res = p.resume + (int64_t)slot * p.resume_stride;
         res_next = res + p.resume_stride / 2;
         for (int64_t f = tid; f < nnzA; f += T) res[f] = 0;
       }
@@ -1131,7 +1160,7 @@ __device__ __noinline__ void dense_row(const SpgemmArgs<V>& p, BlockMeta& bm, in
 // P:785-804): every warp owns a 7 KB region and pulls rows of the bin from a global counter
 // one row ahead, so no warp ever waits at a block barrier for another warp's row (ncu: 33% of
 // the stall samples of the merged-block kernel were barrier waits).  The region is sized to
-// the row (symbolic: products at 66% fill; numeric: exact nnz at 50%), so clearing and the
+// the row (symbolic: 2x products; numeric: 2.5x exact nnz), so clearing and the
 // write-out scan only the slots a row can use.  Rows of the bin (p.rows) or, without global
 // load balancing, every row of A (p.rows == nullptr).
 // -----------------------------------------------------------------------------------
@@ -1145,10 +1174,11 @@ __global__ void __launch_bounds__(kWarpRowThreads, wr_ctas_per_sm(PASS, MODE))
   uint32_t* rk = reinterpret_cast<uint32_t*>(region);
   V* rv = reinterpret_cast<V*>(region + (PASS == 0 ? 0u : wr_num_val_offset<V>(kRegion)));
   const uint32_t cap = PASS == 0 ? wr_sym_cap() : wr_num_cap<V>(kRegion);
+  const int64_t esc_cap = esc_capacity<V>(PASS, kRegion);
   const int64_t n = p.n_entries;
-  constexpr bool kRange = PASS == 1 && MODE != 1;
+  constexpr bool kRange = MODE != 1;
   // row metadata, one field per lane: 0 A_rp[r], 1 A_rp[r+1], 2 prods[r] / C_rp[r], 3 C_rp[r+1],
-  // 4 colmin[r], 5 colmax[r] (one round trip instead of six dependent loads)
+  // 4 colmin[r], 5 colmax[r], 6 prods[r] (numeric) (one round trip instead of seven dependent loads)
   auto fetch = [&](int64_t e, int32_t& row, int64_t& mv) {
     row = -1;
     mv = 0;
@@ -1160,6 +1190,7 @@ __global__ void __launch_bounds__(kWarpRowThreads, wr_ctas_per_sm(PASS, MODE))
       else if (lane == 3 && PASS == 1) mv = p.C_rp[row + 1];
       else if (lane == 4 && kRange) mv = p.colmin[row];   // column range: ordered maps only
       else if (lane == 5 && kRange) mv = p.colmax[row];
+      else if (lane == 6 && PASS == 1 && MODE != 1) mv = p.prods[row];
     }
   };
   // rows are claimed kWarpRowChunk at a time (one same-address atomic per chunk: per-row
@@ -1216,9 +1247,10 @@ __global__ void __launch_bounds__(kWarpRowThreads, wr_ctas_per_sm(PASS, MODE))
     const int64_t m3 = __shfl_sync(0xffffffffu, mv, 3);
     const int32_t cmn = (int32_t)__shfl_sync(0xffffffffu, mv, 4);
     const int32_t cmx = (int32_t)__shfl_sync(0xffffffffu, mv, 5);
+    const int64_t mv_prev6 = mv;
     const int32_t cur = row;
     const int64_t need = PASS == 0 ? m2 : m3 - m2;       // products (symbolic) / exact nnz (numeric)
-    // region: symbolic 1.5x products (66% fill), numeric 2x entries (50% fill), 32-slot multiples
+    // region: symbolic 2x products (<= 50% load), numeric 2.5x entries (<= 40% load), 32-slot multiples
     const uint64_t want = PASS == 0 ? (uint64_t)need * 2 : (uint64_t)need * 5 / 2;
     const uint64_t w32 = (want + 31) & ~(uint64_t)31;
     const uint32_t S = (uint32_t)(w32 < 64 ? 64 : (w32 > cap ? cap : w32));
@@ -1232,7 +1264,15 @@ __global__ void __launch_bounds__(kWarpRowThreads, wr_ctas_per_sm(PASS, MODE))
     row = rown;
     mv = mvn;
     fetch((int64_t)enn, rown, mvn);
-    const int c = warp_row<PASS, V, MODE>(p, rk, rv, S, a0, alen, cmn, cmx, (int32_t)(m3 - m2), m2, &bcur);
+    int c = -1;
+    if (MODE != 1) {
+      // rows whose products are (almost) all distinct columns: counting sort on column buckets
+      // (esc_kernels.cuh); -1 = uneven buckets, the hash map below takes the row
+      const int64_t np = PASS == 0 ? need : __shfl_sync(0xffffffffu, mv_prev6, 6);
+      if (p.esc >= (PASS == 0 ? 2 : 1) && np > 0 && np <= esc_cap && (PASS == 0 || np <= 2 * need))
+        c = esc_row<1, PASS, V>(p, region, kRegion, 0, a0, alen, (int)np, (int)need, cmn, cmx, m2, nullptr, nullptr, 0);
+    }
+    if (c < 0) c = warp_row<PASS, V, MODE>(p, rk, rv, S, a0, alen, cmn, cmx, (int32_t)(m3 - m2), m2, &bcur);
     if (PASS == 0 && lane == 0) p.cnt[cur] = c;
     e = en;
     en = enn;

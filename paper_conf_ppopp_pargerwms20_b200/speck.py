@@ -23,8 +23,19 @@ SPECK_F32, SPECK_F64 = 0, 1
 OPT = {
     "global_lb_symbolic": 0, "global_lb_numeric": 1, "force_accumulator": 2, "dense_window": 3,
     "stage_timing": 4, "validate": 5, "disable_direct": 6, "fixed_group_size": 7, "concurrent_streams": 8,
-    "segments": 9, "warp_rows": 10, "long_bitmap": 11, "bitmap_reuse": 12,
+    "segments": 9, "warp_rows": 10, "long_bitmap": 11, "bitmap_reuse": 12, "kernel_timing": 13,
+    "path_counters": 14, "bucket_sort": 15,
 }
+# speck_kernel_kind_t (kernel id = kind * 16 + configuration)
+KERNEL_KINDS = {1: "analysis", 2: "binning", 3: "scan", 4: "sym_warp", 5: "sym_block", 6: "num_tiny", 7: "num_warp",
+                8: "num_block", 9: "direct", 10: "segments", 11: "long_bitmap", 12: "seg_plan"}
+# speck_path_t
+PATHS = ["sym_warp", "sym_block_hash", "sym_merged", "sym_dense", "sym_dense_multi", "num_tiny", "num_warp_ordered",
+         "num_warp_sorted", "num_block_ordered", "num_block_sorted", "num_merged", "num_dense", "num_dense_multi",
+         "num_direct", "seg_hash", "seg_dense", "seg_windows", "long_bitmap", "long_bitmap_split"]
+PATH_COUNT = 24
+# bin categories of speck_stats_t.bin_* (per pass)
+CATEGORIES = ["empty", "direct", "cfg0", "cfg1", "cfg2", "cfg3", "cfg4", "long", "tiny", "unused"]
 STATUS = {
     0: "SPECK_OK", 1: "SPECK_ERR_INVALID_ARGUMENT", 2: "SPECK_ERR_DIMENSION_MISMATCH", 3: "SPECK_ERR_DTYPE_MISMATCH",
     4: "SPECK_ERR_UNSUPPORTED", 5: "SPECK_ERR_OUT_OF_MEMORY", 6: "SPECK_ERR_CUDA", 7: "SPECK_ERR_NOT_ANALYZED",
@@ -60,13 +71,20 @@ class Stats(ctypes.Structure):
                 ("segments", ctypes.c_int64),
                 ("workspace_bytes", ctypes.c_int64), ("kernel_launches", ctypes.c_int64), ("ms_analysis", ctypes.c_float), ("ms_symbolic_lb", ctypes.c_float),
                 ("ms_symbolic", ctypes.c_float), ("ms_scan", ctypes.c_float), ("ms_numeric_lb", ctypes.c_float),
-                ("ms_numeric", ctypes.c_float)]
+                ("ms_numeric", ctypes.c_float),
+                ("bin_rows", (ctypes.c_int64 * 10) * 2), ("bin_nnza", (ctypes.c_int64 * 10) * 2),
+                ("bin_products", (ctypes.c_int64 * 10) * 2), ("bin_nnzc", ctypes.c_int64 * 10),
+                ("n_kernels", ctypes.c_int32), ("kernel_id", ctypes.c_int32 * 64), ("kernel_bin", ctypes.c_int32 * 64),
+                ("kernel_ms", ctypes.c_float * 64), ("path_rows", ctypes.c_int64 * PATH_COUNT)]
 
     def as_dict(self):
-        d = {}
-        for name, _ in self._fields_:
-            v = getattr(self, name)
-            d[name] = list(v) if hasattr(v, "__len__") else v
+        def conv(v):
+            return [conv(x) for x in v] if hasattr(v, "__len__") else v
+        d = {name: conv(getattr(self, name)) for name, _ in self._fields_}
+        n = d["n_kernels"]
+        d["kernels"] = [{"kind": KERNEL_KINDS.get(i >> 4, str(i >> 4)), "cfg": i & 15, "bin": b, "ms": ms}
+                        for i, b, ms in zip(d["kernel_id"][:n], d["kernel_bin"][:n], d["kernel_ms"][:n])]
+        d["paths"] = dict(zip(PATHS, d["path_rows"]))
         return d
 
 

@@ -53,7 +53,7 @@ def test_stats_struct_layout():
     import paper_conf_ppopp_pargerwms20_b200 as sp
     txt = open(HEADER).read()
     body = txt[txt.index("typedef struct {\n  int64_t products;"):txt.index("} speck_stats_t;")]
-    names = re.findall(r"\b([a-z_]+)(?:\[\d+\])?\s*[;,]", re.sub(r"/\*.*?\*/", "", body, flags=re.S))
+    names = re.findall(r"\b([a-z_]+)(?:\[[A-Z_\d]+\])*\s*[;,]", re.sub(r"/\*.*?\*/", "", body, flags=re.S))
     assert [n for n, _ in sp.Stats._fields_] == names
 
 

@@ -345,3 +345,89 @@ def test_group_size_properties():
         assert T // g <= max(nnzA, 1) or g == T
     # Fig. 1 situation: avg len 3 -> g starts at 4; iter_max = 2, n_rows = 4/2 = 2 -> keep 4
     assert oracle.group_size(8, 4, 12, 7) == 4
+
+
+def test_group_size_sqrt_branches_hand_derived():
+    """Reading R9, both sqrt branches and the final k <= NNZ_A clamp, each value
+    derived by hand from the formula (not by calling the oracle):
+    (a) T=256, nnzA=64, maxlen=4288, prods=4351: avg 67.98 -> g=64, k=4, iter_max=ceil(4288/64)=67,
+        n_rows=16; 67 > 2*16 -> g = 64*sqrt(67/32) = 92.6 -> closest power of two in linear
+        distance: 64 (28.6 < 35.4).  Dropping the sqrt gives 134 -> 128; log-distance rounding
+        gives 128; dropping the factor 2 gives 64*sqrt(67/16) = 131 -> 128.
+    (b) T=256, nnzA=1024, maxlen=16, prods=4096: avg 4 -> g=4, k=64, iter_max=4, n_rows=16;
+        16 > 2*4 -> g = 4*sqrt(4/16) = 2.  Without the sqrt: 4*4/16 = 1.
+    (c) T=1024, nnzA=3, maxlen=2, prods=6: g=2, k=512, iter_max=1, n_rows=3/512; first branch
+        -> 2*sqrt(1/(2*3/512)) = 18.5 -> 16; k = 64 > nnzA = 3 -> k = 2 (largest pow2 <= 3),
+        g = 1024/2 = 512."""
+    assert oracle.group_size(256, 64, 4351, 4288) == 64
+    assert oracle.group_size(256, 1024, 4096, 16) == 2
+    assert oracle.group_size(1024, 3, 6, 2) == 512
+    # neither branch: (T=256, nnzA=64, maxlen=64, prods=4096): g=64, k=4, iter_max=1, n_rows=16
+    # -> 16 > 2 -> g = 64*sqrt(1/16) = 16
+    assert oracle.group_size(256, 64, 4096, 64) == 16
+
+
+def test_check_csr_rejects_each_violation():
+    """oracle_check_csr (columns strictly ascending inside a row, in [0, ncols)) returns
+    the first offending row for each kind of violation and -1 only for valid CSR."""
+    rp = np.array([0, 2, 4, 6], np.int64)
+    ok = np.array([0, 3, 1, 2, 0, 4], np.int32)
+    assert oracle.check_csr(3, 5, rp, ok) == -1
+    assert oracle.check_csr(3, 5, rp, np.array([0, 3, 2, 1, 0, 4], np.int32)) == 1     # unsorted row 1
+    assert oracle.check_csr(3, 5, rp, np.array([0, 3, 1, 2, 4, 4], np.int32)) == 2     # duplicate in row 2
+    assert oracle.check_csr(3, 5, rp, np.array([0, 5, 1, 2, 0, 4], np.int32)) == 0     # column == ncols
+    assert oracle.check_csr(3, 5, rp, np.array([0, 3, -1, 2, 0, 4], np.int32)) == 1    # negative column
+    assert oracle.check_csr(3, 5, np.array([0, 2, 1, 6], np.int64), ok) == 1           # decreasing row_ptr
+    assert oracle.check_csr(0, 5, np.array([0], np.int64), np.zeros(0, np.int32)) == -1
+
+
+# ----------------------------------------------------------------- the comparator itself
+def _cmp_case():
+    rp = np.array([0, 2, 3], np.int64)
+    col = np.array([1, 4, 0], np.int32)
+    val = np.array([1.0, -2.0, 0.0])
+    scale = np.array([1.0, 2.0, 0.0])
+    return rp, col, val, scale
+
+
+def test_compare_accepts_exact_and_within_tolerance():
+    rp, col, val, scale = _cmp_case()
+    assert oracle.compare(rp, col, val, rp, col, val, scale, 1e-5)["ok"]
+    g = val.copy(); g[0] += 0.5e-5 * scale[0]; g[2] = -0.0        # half of tol·s; -0 where s = 0
+    assert oracle.compare(rp + 7, col, g, rp, col, val, scale, 1e-5)["ok"]   # offsets compared relative
+
+
+@pytest.mark.parametrize("kind", ["nan", "inf", "ulp_past_tol", "nonzero_where_s0", "swapped_col",
+                                  "off_by_one_rowptr", "short_arrays"])
+def test_compare_rejects(kind):
+    """Every parity claim rests on oracle.compare: each plausible GPU error must fail it."""
+    rp, col, val, scale = _cmp_case()
+    g_rp, g_col, g_val = rp.copy(), col.copy(), val.copy()
+    if kind == "nan":
+        g_val[1] = np.nan
+    elif kind == "inf":
+        g_val[0] = np.inf
+    elif kind == "ulp_past_tol":
+        g_val = np.array([0.0, -2.0, 0.0]); r = np.array([0.0, -2.0, 0.0]); s = np.array([1.0, 2.0, 0.0])
+        g_val[0] = np.nextafter(1e-5, 1.0)                          # one ulp beyond tol·s = 1e-5
+        res = oracle.compare(rp, col, g_val, rp, col, r, s, 1e-5)
+        assert not res["ok"] and res["n_viol"] == 1 and res["first_bad"] == 0
+        return
+    elif kind == "nonzero_where_s0":
+        g_val[2] = 1e-300
+    elif kind == "swapped_col":
+        g_col[[0, 1]] = g_col[[1, 0]]
+    elif kind == "off_by_one_rowptr":
+        g_rp[1] += 1
+    elif kind == "short_arrays":
+        g_col, g_val = g_col[:2], g_val[:2]
+    res = oracle.compare(g_rp, g_col, g_val, rp, col, val, scale, 1e-5)
+    assert not res["ok"], (kind, res)
+    if kind in ("nan", "inf"):
+        assert res["n_nonfinite"] == 1
+
+
+def test_compare_nan_even_with_huge_tolerance():
+    rp, col, val, scale = _cmp_case()
+    g = val.copy(); g[0] = np.nan
+    assert not oracle.compare(rp, col, g, rp, col, val, scale, 1e300)["ok"]

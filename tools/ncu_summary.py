@@ -56,7 +56,7 @@ def main(rep, launch=0):
     for o in sorted(out, reverse=True)[:20]:
         print(f"  {100 * o[0] / ts:5.1f}% stalls {100 * o[1] / ti:5.1f}% inst  {o[2]}:{o[3]}  {o[4]}")
     print("top source lines by executed warp instructions:")
-    for o in sorted(out, key=lambda x: -x[1])[:15]:
+    for o in sorted(out, key=lambda x: -x[1])[:40]:
         print(f"  {100 * o[0] / ts:5.1f}% stalls {100 * o[1] / ti:5.1f}% inst  {o[2]}:{o[3]}  {o[4]}")
 
 
