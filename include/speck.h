@@ -97,7 +97,7 @@ typedef enum {
                                        atomics per row — tests and diagnostics only [0] */
   SPECK_OPT_BUCKET_SORT = 15        /* rows whose products are mostly distinct columns use a counting sort on
                                        column buckets instead of the hash map: 0 off, 1 numeric rows, 2 numeric
-                                       and symbolic rows [2] */
+                                       and symbolic rows [1] */
 } speck_option_t;
 /* Changing any option except STAGE_TIMING, CONCURRENT_STREAMS, GLOBAL_LB_NUMERIC, VALIDATE,
  * KERNEL_TIMING and PATH_COUNTERS after speck_analyze invalidates the analysis: the next
@@ -140,6 +140,10 @@ typedef enum {
   SPECK_PATH_SEG_WINDOWS = 16,    /* long row, sequential dense windows (per job) */
   SPECK_PATH_LONG_BITMAP = 17,    /* long row, bitmap + rank CTA */
   SPECK_PATH_LONG_BITMAP_SPLIT = 18,/* long row, bitmap kept by the symbolic step, split over CTAs (per CTA) */
+  SPECK_PATH_SYM_ESC = 19,        /* symbolic bucket counting sort (esc_kernels.cuh) */
+  SPECK_PATH_NUM_ESC = 20,        /* numeric bucket counting sort, no repeated column */
+  SPECK_PATH_NUM_ESC_DUP = 21,    /* numeric bucket counting sort with repeated columns */
+  SPECK_PATH_ESC_FALLBACK = 22,   /* bucket counting sort abandoned (uneven buckets): hash map instead */
   SPECK_PATH_COUNT = 24
 } speck_path_t;
 
@@ -203,6 +207,34 @@ speck_status_t speck_analyze(speck_handle_t handle, const speck_csr_t* A, const 
 speck_status_t speck_spgemm(speck_handle_t handle, const speck_csr_t* A, const speck_csr_t* B,
                             const int64_t* C_row_ptr, int32_t* C_col_idx, void* C_values,
                             speck_stream_t stream);
+
+/* Memory-bounded numeric phase (the paper's future work "partial
+ * multiplications of large matrices on single GPUs"): after speck_analyze, the
+ * numeric phase of the rows [r0, r1) only.  C_row_ptr is the full array speck_analyze wrote;
+ * C_col_part / C_val_part (device, caller-owned) hold the chunk's C_row_ptr[r1] - C_row_ptr[r0]
+ * entries: entry t of row i goes to index C_row_ptr[i] - C_row_ptr[r0] + t.  Calls for different
+ * ranges may follow one speck_analyze in any order; together they produce exactly the entries
+ * speck_spgemm would.  One small D2H synchronisation per call (the chunk's bin ranges); the
+ * numeric work is asynchronous.  Invalid ranges -> SPECK_ERR_INVALID_ARGUMENT. */
+speck_status_t speck_spgemm_rows(speck_handle_t handle, const speck_csr_t* A, const speck_csr_t* B,
+                                 const int64_t* C_row_ptr, int64_t r0, int64_t r1, int32_t* C_col_part,
+                                 void* C_val_part, speck_stream_t stream);
+
+/* Device CSR transpose: T = Aᵀ in sorted CSR, for the paper's A·Aᵀ protocol
+ * ("rectangular matrices ... multiplied with their transpose", Aᵀ precomputed) and
+ * the AMG restriction R = Pᵀ.  T is A.cols x A.rows: T_row_ptr device int64 [A.cols + 1],
+ * T_col_idx int32 [A.nnz], T_values [A.nnz] of A's dtype (NULL exactly when A.values is NULL),
+ * all caller-owned.  Values are moved bit for bit; every row of T is sorted.  Synchronises
+ * `stream` (row-length statistics are read back to size the sort). */
+speck_status_t speck_transpose(speck_handle_t handle, const speck_csr_t* A, int64_t* T_row_ptr, int32_t* T_col_idx,
+                               void* T_values, speck_stream_t stream);
+
+/* Row chunks for a memory budget: splits [0, rows) of the analysed C (C_row_ptr, device) into
+ * consecutive ranges of fewer than max_nnz entries each (some may be empty).  Writes
+ * bounds[0..n] (host, int64, n <= max_parts) and *n_parts = n.  max_nnz must exceed the longest
+ * row of C (else SPECK_ERR_INVALID_ARGUMENT).  Synchronous. */
+speck_status_t speck_row_chunks(speck_handle_t handle, const int64_t* C_row_ptr, int64_t rows, int64_t max_nnz,
+                                int64_t* bounds, int64_t max_parts, int64_t* n_parts);
 
 /* Row analysis only (Alg. 1).  Per row i of A (device arrays, [A.rows]):
  *   prods[i]  = Σ_{k ∈ A_i} |B_k|           maxlen[i] = max_k |B_k|

@@ -37,7 +37,8 @@ def needs_build() -> bool:
 def build(force: bool = False, verbose: bool = False) -> str:
     if not force and not needs_build():
         return LIB
-    cmd = [nvcc(), *NVCC_FLAGS, "-o", LIB + ".tmp", *SOURCES]
+    extra = os.environ.get("SPECK_NVCC_EXTRA", "").split()      # experiments only (e.g. -DSPECK_ESC_LAMBDA=1)
+    cmd = [nvcc(), *NVCC_FLAGS, *extra, "-o", LIB + ".tmp", *SOURCES]
     res = subprocess.run(cmd, capture_output=True, text=True)
     log = res.stdout + res.stderr
     with open(os.path.join(HERE, "build.log"), "w") as f:

@@ -29,8 +29,13 @@
 
 namespace speck {
 
-constexpr int kEscLambda = 4;        // target products per bucket
-constexpr int kEscMaxBucket = 96;    // a row whose largest bucket exceeds this goes back to the hash map
+#ifndef SPECK_ESC_LAMBDA
+#define SPECK_ESC_LAMBDA 2
+#endif
+constexpr int kEscLambda = SPECK_ESC_LAMBDA;   // target products per bucket
+// a row whose largest bucket exceeds this goes back to the hash map: clustered columns (stencil
+// rows: many products on few columns) would make the in-bucket ranking quadratic
+constexpr int kEscMaxBucket = 8 * kEscLambda + 16;
 constexpr uint32_t kEscDropBit = 0x80000000u;   // marks a non-first duplicate (columns are < 2^31)
 
 template <typename V>
@@ -40,6 +45,13 @@ template <typename V>
 __host__ __device__ inline int64_t esc_capacity(int pass, int64_t bytes) {
   return (bytes - 320) * kEscLambda / ((int64_t)esc_entry_bytes<V>(pass) * kEscLambda + 8);
 }
+// rank of k among keys[s, en) (keys < k), two keys per iteration
+__device__ __forceinline__ int esc_rank(const uint32_t* keys, int s, int en, uint32_t k) {
+  int r = 0, j = s;
+  for (; j + 2 <= en; j += 2) r += (keys[j] < k) + (keys[j + 1] < k);
+  if (j < en) r += keys[j] < k;
+  return r;
+}
 
 template <int NW>
 __device__ __forceinline__ void esc_sync() {
@@ -48,8 +60,19 @@ __device__ __forceinline__ void esc_sync() {
 
 // Products of A_i (NZ [a0, a0 + alen)) for warp wi of nw (a power of two): chunks of 32 products
 // rotate over the warps across batches.  f(col, a*b, active) is called by all 32 lanes.
+// `pre` (optional): the row's first batch, loaded ahead by the caller (lane f: B row start /
+// length and a of the row's f-th NZ).
+template <typename V>
+struct PreBatch {
+  int64_t bst = 0;
+  int blen = 0;
+  V a = V(0);
+  bool valid = false;
+};
+
 template <int PASS, typename V, int U, typename F>
-__device__ __forceinline__ void expand_esc(const SpgemmArgs<V>& p, int64_t a0, int alen, int wi, int nw, F&& f) {
+__device__ __forceinline__ void expand_esc(const SpgemmArgs<V>& p, int64_t a0, int alen, int wi, int nw, F&& f,
+                                           const PreBatch<V>* pre = nullptr) {
   const int lane = lane_id();
   int rot = 0;
   for (int b0 = 0; b0 < alen; b0 += 32) {
@@ -57,7 +80,11 @@ __device__ __forceinline__ void expand_esc(const SpgemmArgs<V>& p, int64_t a0, i
     int64_t bst = 0;
     int blen = 0;
     V a = V(0);
-    if (fi < alen) {
+    if (pre && b0 == 0 && pre->valid) {
+      bst = pre->bst;
+      blen = pre->blen;
+      a = pre->a;
+    } else if (fi < alen) {
       const int32_t kc = p.A_col[a0 + fi];
       if (PASS == 1) a = __ldg(p.A_val + a0 + fi);
       bst = p.B_rp[kc];
@@ -164,7 +191,7 @@ __device__ __forceinline__ int esc_scan(int* bc, int NB, int wi, int* red) {
 //   PASS 1: writes the row sorted at C[cbase, cbase + cnt); returns cnt, or -1 (fallback).
 // chist (symbolic, may be null): distinct columns per 2^chunk_shift-column chunk (long rows).
 template <int NW, int PASS, typename V>
-__device__ int esc_row(const SpgemmArgs<V>& p, unsigned char* region, uint32_t region_bytes, int wi, int64_t a0,
+__device__ __forceinline__ int esc_row(const SpgemmArgs<V>& p, unsigned char* region, uint32_t region_bytes, int wi, int64_t a0,
                        int alen, int n, int cnt, int32_t cmin, int32_t cmax, int64_t cbase, int* red, int* chist,
                        int chunk_shift) {
   const int lane = lane_id();
@@ -190,7 +217,11 @@ __device__ int esc_row(const SpgemmArgs<V>& p, unsigned char* region, uint32_t r
   });
   esc_sync<NW>();
   const int mx = esc_scan<NW>(bc, NB, wi, red);
-  if (mx > kEscMaxBucket) return -1;
+  if (mx > kEscMaxBucket) {
+    if (t == 0) count_path(p.paths, SPECK_PATH_ESC_FALLBACK);
+    return -1;
+  }
+  if (t == 0) count_path(p.paths, PASS == 0 ? SPECK_PATH_SYM_ESC : n == cnt ? SPECK_PATH_NUM_ESC : SPECK_PATH_NUM_ESC_DUP);
   // ---- S: append (col, a*b) to its bucket -----------------------------------------------------
   expand_esc<PASS, V, 2>(p, a0, alen, wi, NW, [&](uint32_t col, V v, bool act) {
     if (act) {
@@ -229,8 +260,7 @@ __device__ int esc_row(const SpgemmArgs<V>& p, unsigned char* region, uint32_t r
       const uint32_t k = keys[e];
       const uint32_t b = home(k);
       const int s = b ? bc[b - 1] : 0, en = bc[b];
-      int r = 0;
-      for (int j = s; j < en; ++j) r += keys[j] < k;
+      const int r = esc_rank(keys, s, en, k);
       p.C_col[cbase + s + r] = (int32_t)k;
       p.C_val[cbase + s + r] = vals[e];
     }
@@ -271,8 +301,7 @@ __device__ int esc_row(const SpgemmArgs<V>& p, unsigned char* region, uint32_t r
     if (k & kEscDropBit) continue;
     const uint32_t b = home(k);
     const int s = b ? bc[b - 1] : 0, en = bc[b];
-    int r = 0;
-    for (int j = s; j < en; ++j) r += keys[j] < k;     // dropped keys have the top bit set: never smaller
+    const int r = esc_rank(keys, s, en, k);          // dropped keys have the top bit set: never smaller
     const int64_t o = cbase + dc[b] + r;
     p.C_col[o] = (int32_t)k;
     p.C_val[o] = vals[e];

@@ -291,6 +291,48 @@ __global__ void __launch_bounds__(kBinTile) k_bin_scatter(const int64_t* __restr
 }
 
 // ------------------------------------------------------------------------------------
+// Row-range numeric (speck_spgemm_rows): the bins keep CSR order, so the rows of [r0, r1) form
+// one contiguous sub-range of every category's bin.  Thread c finds category c's sub-range by
+// binary search; out[2c], out[2c+1] = begin / end positions in `bins`; out[2 CAT_COUNT],
+// out[2 CAT_COUNT + 1] = C_rp[r0], C_rp[r1] (the chunk's entries).
+// ------------------------------------------------------------------------------------
+struct CatStarts { int64_t s[CAT_COUNT + 1]; };
+__global__ void k_bin_range(const int32_t* __restrict__ bins, CatStarts cs, int64_t r0, int64_t r1,
+                            const int64_t* __restrict__ C_rp, int64_t* __restrict__ out) {
+  const int c = threadIdx.x;
+  if (c < CAT_COUNT) {
+    auto lb = [&](int64_t x) {
+      int64_t l = cs.s[c], h = cs.s[c + 1];
+      while (l < h) {
+        const int64_t mid = (l + h) >> 1;
+        if ((int64_t)bins[mid] < x) l = mid + 1; else h = mid;
+      }
+      return l;
+    };
+    out[2 * c] = lb(r0);
+    out[2 * c + 1] = lb(r1);
+  }
+  if (c == 0) { out[2 * CAT_COUNT] = C_rp[r0]; out[2 * CAT_COUNT + 1] = C_rp[r1]; }
+}
+
+// Memory-bounded chunks (speck_row_chunks): bound_j = first row whose C offset is >= j * step,
+// j = 1 .. parts-1 (step = max_nnz - longest row), so every chunk holds < max_nnz entries.
+__global__ void k_chunk_bounds(const int64_t* __restrict__ C_rp, int64_t m, int64_t step, int64_t parts,
+                               int64_t* __restrict__ out) {
+  const int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (j > parts) return;
+  if (j == 0) { out[0] = 0; return; }
+  if (j == parts) { out[parts] = m; return; }
+  const int64_t x = j * step;
+  int64_t l = 0, h = m;
+  while (l < h) {
+    const int64_t mid = (l + h) >> 1;
+    if (C_rp[mid] < x) l = mid + 1; else h = mid;
+  }
+  out[j] = l;
+}
+
+// ------------------------------------------------------------------------------------
 // Single-pass exclusive scan of int64 (decoupled look-back), used for the C row offsets
 // and for the bin offsets.  out[0..n] with out[n] = total.  Each CTA takes
 // a dynamic tile id so predecessors are always scheduled before successors.

@@ -173,7 +173,7 @@ __device__ int64_t dense_window_pass(const SpgemmArgs<V>& p, int64_t a0, int ale
 // One CTA of configuration kSegCfg (2 CTAs/SM) per job.
 template <typename V>
 __global__ void __launch_bounds__(kCfgThreads[kSegCfg], 1024 / kCfgThreads[kSegCfg])
-    k_segments(SpgemmArgs<V> p, const Seg* __restrict__ segs) {
+    k_segments(const __grid_constant__ SpgemmArgs<V> p, const Seg* __restrict__ segs) {
   constexpr int CFG = kSegCfg;
   constexpr int T = kCfgThreads[CFG];
   constexpr int NW = T / 32;
@@ -182,9 +182,13 @@ __global__ void __launch_bounds__(kCfgThreads[kSegCfg], 1024 / kCfgThreads[kSegC
   __shared__ int s_wrap;
   const int tid = threadIdx.x;
   const Seg sg = segs[blockIdx.x];
+  if (sg.row < p.row_lo || sg.row >= p.row_hi) return;    // row-range numeric: another chunk's row
   const int64_t a0 = p.A_rp[sg.row];
   const int alen = (int)(p.A_rp[sg.row + 1] - a0);
   const uint32_t lo = (uint32_t)sg.col_lo, hi = (uint32_t)sg.col_hi, range = hi - lo;
+  if (tid == 0)
+    count_path(p.paths, sg.dense == SEG_HASH ? SPECK_PATH_SEG_HASH : sg.dense == SEG_DENSE ? SPECK_PATH_SEG_DENSE
+                                                                                         : SPECK_PATH_SEG_WINDOWS);
 
   if (sg.dense == SEG_HASH) {
     uint32_t* keys = reinterpret_cast<uint32_t*>(smem);
@@ -272,13 +276,14 @@ constexpr int kBitmapThreads = 1024;
 constexpr int64_t kBitmapMaxCols = (int64_t)(kCfgMapBytes[kNumCfg - 1] / 196) * 1024;
 
 template <typename V>
-__global__ void __launch_bounds__(kBitmapThreads, 1) k_long_bitmap(SpgemmArgs<V> p, SegPlanArgs a) {
+__global__ void __launch_bounds__(kBitmapThreads, 1) k_long_bitmap(const __grid_constant__ SpgemmArgs<V> p, const __grid_constant__ SegPlanArgs a) {
   constexpr int T = kBitmapThreads, NW = T / 32;
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ int64_t part[NW + 1];
   __shared__ LongList<V> longs;
   const int ci = blockIdx.x / a.split_max, piece = blockIdx.x % a.split_max;
   const int32_t row = a.cand[ci];
+  if (row < p.row_lo || row >= p.row_hi) return;           // row-range numeric: another chunk's row
   const int64_t ob = a.C_rp[row], cnt = a.C_rp[row + 1] - ob;
   if (cnt <= a.limit || !bitmap_row(a, row)) return;
   const long long bmo = a.bm_pool ? a.bm_off[ci] : -1ll;
@@ -292,6 +297,7 @@ __global__ void __launch_bounds__(kBitmapThreads, 1) k_long_bitmap(SpgemmArgs<V>
   }
   if (piece >= pieces) return;
   const int tid = threadIdx.x, lane = lane_id(), wp = warp_id();
+  if (tid == 0) count_path(p.paths, pieces == 1 ? SPECK_PATH_LONG_BITMAP : SPECK_PATH_LONG_BITMAP_SPLIT);
   const uint32_t lo = (uint32_t)a.colmin[row] & ~31u;
   const int W = (int)(((int64_t)a.colmax[row] + 1 - lo + 31) / 32);
   const int G = (W + 31) / 32;                                   // 32-word groups

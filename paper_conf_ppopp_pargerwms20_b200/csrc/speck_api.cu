@@ -16,6 +16,7 @@
 #include "plan_kernels.cuh"
 #include "spgemm_kernels.cuh"
 #include "segment_kernels.cuh"
+#include "transpose_kernels.cuh"
 
 #define SPECK_VERSION "speck-b200 0.1.0 (sm_100a)"
 
@@ -38,6 +39,8 @@ constexpr int kPinSymCat = 16;     // [CAT_COUNT + 1] bin offsets
 constexpr int kPinBinSums = 64;    // [2][CAT_COUNT][3] per-bin sums (nnzA, products, nnzC)
 // `small` device scratch layout (bytes)
 constexpr int kSmallBinSums = 3072;   // unsigned long long [2][CAT_COUNT][3]
+constexpr int kSmallRange = 3584;     // int64 [2 CAT_COUNT + 1] (speck_spgemm_rows)
+constexpr int kPinRange = 128;        // pinned words for the same
 
 }  // namespace speck
 
@@ -50,7 +53,7 @@ struct speck_handle_s {
   std::string err;
   // options
   int64_t opt_lb_sym = -1, opt_lb_num = -1, opt_force_acc = 0, opt_dense_window = 0, opt_timing = 0, opt_validate = 0,
-          opt_disable_direct = 0, opt_fixed_g = 0, opt_streams = 4, opt_esc = 2;
+          opt_disable_direct = 0, opt_fixed_g = 0, opt_streams = 4, opt_esc = 1;
   // workspace
   Buf prods, maxlen, colmin, colmax, cnt, hist, hist_off, bins, stats, scan_status, resume, small, ana_long, binfo;
   unsigned long long* h_pinned = nullptr;  // pinned readback area (kPinnedWords x u64)
@@ -67,6 +70,7 @@ struct speck_handle_s {
   speck_stats_t st = {};
   int lb_num = 0;
   bool numeric_pending = false;
+  bool num_binned = false;   // numeric bins of the current analysis scattered (speck_spgemm_rows)
   int64_t launches = 0;  // kernels launched by this handle (cumulative)
   // long-row segments
   int64_t opt_segments = 1;
@@ -79,7 +83,7 @@ struct speck_handle_s {
   bool seg_enabled = false;
   int seg_shift = 15, nchunks = 0;
   int64_t long_thr = INT64_MAX, n_cand = 0, n_segs = 0, cand_start = 0;
-  Buf chunk_cnt, cand, nseg, seg_off, segs;
+  Buf chunk_cnt, cand, nseg, seg_off, segs, chunks, tr_cnt, tr_list, tr_col, tr_val;
   // SPECK_OPT_KERNEL_TIMING: one event pair per launch of the current analyze/spgemm pair
   int64_t opt_ktime = 0, opt_paths = 0;
   cudaEvent_t kt_ev[2 * kMaxTimed] = {};
@@ -172,7 +176,8 @@ int64_t ws_bytes(speck_handle_t h) {
   return (int64_t)(h->prods.cap + h->maxlen.cap + h->colmin.cap + h->colmax.cap + h->cnt.cap + h->hist.cap +
                    h->hist_off.cap + h->bins.cap + h->stats.cap + h->scan_status.cap + h->resume.cap + h->small.cap +
                    h->ana_long.cap + h->chunk_cnt.cap + h->cand.cap + h->nseg.cap + h->seg_off.cap + h->segs.cap +
-                   h->bm_pool.cap + h->bm_off.cap + h->binfo.cap);
+                   h->bm_pool.cap + h->bm_off.cap + h->binfo.cap + h->paths.cap + h->chunks.cap +
+                   h->tr_cnt.cap + h->tr_list.cap + h->tr_col.cap + h->tr_val.cap);
 }
 
 speck_status_t check_csr(speck_handle_t h, const speck_csr_t* M, const char* name, bool need_values) {
@@ -272,8 +277,10 @@ speck_status_t set_smem_attrs(speck_handle_t h) {
     for (int pass = 0; pass < 2; ++pass)
       CK(cudaFuncSetAttribute(spgemm_fn<V>(c, pass), cudaFuncAttributeMaxDynamicSharedMemorySize, kCfgMapBytes[c]));
   CK(cudaFuncSetAttribute(k_segments<V>, cudaFuncAttributeMaxDynamicSharedMemorySize, kCfgMapBytes[kSegCfg]));
+  CK(cudaFuncSetAttribute(k_tr_sort_block<V>, cudaFuncAttributeMaxDynamicSharedMemorySize, kTrSmemSort * (4 + (int)sizeof(V))));
   CK(cudaFuncSetAttribute(k_long_bitmap<V>, cudaFuncAttributeMaxDynamicSharedMemorySize, kCfgMapBytes[kNumCfg - 1]));
   CK(cudaFuncSetAttribute(k_warp_rows<0, V, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytesSym * (kWarpRowThreads / 32)));
+  CK(cudaFuncSetAttribute(k_warp_rows<0, V, 3>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytesSym * (kWarpRowThreads / 32)));
   CK(cudaFuncSetAttribute(k_warp_rows<1, V, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytes * (kWarpRowThreads / 32)));
   CK(cudaFuncSetAttribute(k_warp_rows<1, V, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytesTiny * (kWarpRowThreads / 32)));
   CK(cudaFuncSetAttribute(k_warp_rows<1, V, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytes * (kWarpRowThreads / 32)));
@@ -325,7 +332,8 @@ speck_status_t launch_warp_rows(speck_handle_t h, int pass, const SpgemmArgs<V>&
   const size_t smem = (size_t)wr_region_bytes(pass, md) * (kWarpRowThreads / 32);
   const int kt = kt_begin(h, s, pass == 0 ? SPECK_KERNEL_SYM_WARP : md == 1 ? SPECK_KERNEL_NUM_TINY : SPECK_KERNEL_NUM_WARP,
                           md, bin);
-  if (pass == 0) k_warp_rows<0, V, 0><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
+  if (pass == 0 && a.esc >= 2) k_warp_rows<0, V, 3><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
+  else if (pass == 0) k_warp_rows<0, V, 0><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
   else if (mode == 1) k_warp_rows<1, V, 1><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
   else if (mode == 2) k_warp_rows<1, V, 2><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
   else k_warp_rows<1, V, 0><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
@@ -402,6 +410,9 @@ SpgemmArgs<V> base_args(speck_handle_t h, const speck_csr_t* A, const speck_csr_
   a.dense_window_cap = h->opt_dense_window;
   a.fixed_g = (int)h->opt_fixed_g;
   a.esc = (int)h->opt_esc;
+  a.paths = h->opt_paths ? static_cast<unsigned long long*>(h->paths.p) : nullptr;
+  a.row_lo = 0;
+  a.row_hi = INT64_MAX;
   a.cnt = static_cast<int64_t*>(h->cnt.p);
   a.resume = static_cast<int32_t*>(h->resume.p);
   a.resume_stride = 2 * std::max<int64_t>(h->max_nnza, 1);   // two buffers (cur / next) per SM slot
@@ -443,8 +454,9 @@ SegPlanArgs seg_plan_args(speck_handle_t h, const int64_t* C_rp) {
 // Launch one pass (symbolic pass=0 / numeric pass=1) either over the bins (LB on) or over
 // fixed groups of consecutive rows (LB off).
 template <typename V>
-speck_status_t run_pass(speck_handle_t h, int pass, int lb, const int64_t* cat_start, SpgemmArgs<V> a, int64_t need_max,
-                        const BinParams& bp, cudaStream_t s) {
+speck_status_t run_pass(speck_handle_t h, int pass, int lb, const int64_t* cat_beg, const int64_t* cat_end,
+                        SpgemmArgs<V> a, int64_t need_max, const BinParams& bp, cudaStream_t s, int64_t c_off = 0,
+                        int64_t c_len = -1) {
   const int64_t m = a.m;
   if (!lb) {
     // no load balancing: one configuration with room for R rows of the longest size.
@@ -492,7 +504,8 @@ speck_status_t run_pass(speck_handle_t h, int pass, int lb, const int64_t* cat_s
     sa0 = seg_plan_args<V>(h, a.C_rp);
     if (sa0.bitmap_cols > 0 && sa0.bm_pool && h->n_cand <= kSplitMaxCand) {
       sa0.split_max = kSplitPieces;
-      CK(cudaMemsetAsync(a.C_val, 0, (size_t)h->nnz_c * sizeof(V), s));
+      // only this call's rows (the whole C, or a chunk's range of it)
+      CK(cudaMemsetAsync(a.C_val + c_off, 0, (size_t)(c_len < 0 ? h->nnz_c : c_len) * sizeof(V), s));
     }
   }
   if ((st = fork(h, s, ns))) return st;
@@ -519,10 +532,10 @@ speck_status_t run_pass(speck_handle_t h, int pass, int lb, const int64_t* cat_s
   // largest configurations first so long rows start early
   for (int c = kNumCfg - 1; c >= 0; --c) {
     const int cat = CAT_CFG0 + c;
-    const int64_t n = cat_start[cat + 1] - cat_start[cat];
+    const int64_t n = cat_end[cat] - cat_beg[cat];
     if (n <= 0) continue;
     SpgemmArgs<V> b = a;
-    b.rows = bins + cat_start[cat];
+    b.rows = bins + cat_beg[cat];
     b.n_entries = n;
     if (c == 0 && h->opt_warp_rows) {
       st = launch_warp_rows<V>(h, pass, b, h->streams[si], pass == 1 ? 2 : 0, pass * 16 + cat);
@@ -554,28 +567,28 @@ speck_status_t run_pass(speck_handle_t h, int pass, int lb, const int64_t* cat_s
     if (st) return st;
     si = (si + 1) % ns;
   }
-  if (pass == 1 && cat_start[CAT_TINY + 1] > cat_start[CAT_TINY]) {
+  if (pass == 1 && cat_end[CAT_TINY] > cat_beg[CAT_TINY]) {
     SpgemmArgs<V> b = a;
-    b.rows = bins + cat_start[CAT_TINY];
-    b.n_entries = cat_start[CAT_TINY + 1] - cat_start[CAT_TINY];
+    b.rows = bins + cat_beg[CAT_TINY];
+    b.n_entries = cat_end[CAT_TINY] - cat_beg[CAT_TINY];
     st = launch_warp_rows<V>(h, pass, b, h->streams[si], 1, 16 + CAT_TINY);
     if (st) return st;
     si = (si + 1) % ns;
   }
   if (pass == 1) {
-    const int64_t n = cat_start[CAT_DIRECT + 1] - cat_start[CAT_DIRECT];
+    const int64_t n = cat_end[CAT_DIRECT] - cat_beg[CAT_DIRECT];
     if (n > 0) {
       // GD lanes per row: average length of B rows
       const double avg = h->B_rows > 0 ? (double)h->B_nnz / (double)h->B_rows : 1.0;
       const int gd = pow2_clamp(avg, 1, 32);
       const int64_t rows_per_cta = 256 / gd;
       const unsigned grid = (unsigned)std::min<int64_t>((n + rows_per_cta - 1) / rows_per_cta, (int64_t)h->num_sms * 16);
-      const int32_t* rows = bins + cat_start[CAT_DIRECT];
+      const int32_t* rows = bins + cat_beg[CAT_DIRECT];
       cudaStream_t ds = h->streams[si];
       const int kt = kt_begin(h, ds, SPECK_KERNEL_DIRECT, 0, 16 + CAT_DIRECT);
 #define SPECK_DIRECT(GD)                                                                                   \
   k_direct<V, GD><<<grid, 256, 0, ds>>>(rows, n, a.A_rp, a.A_col, a.A_val, a.B_rp, a.B_col, a.B_val, a.C_rp, \
-                                        a.C_col, a.C_val)
+                                        a.C_col, a.C_val, a.paths)
       switch (gd) {
         case 1: SPECK_DIRECT(1); break;
         case 2: SPECK_DIRECT(2); break;
@@ -756,7 +769,7 @@ speck_status_t analyze_impl(speck_handle_t h, const speck_csr_t* A, const speck_
   }
   if ((st = timing_mark(h, 2, s))) return st;
   // ---- 3. symbolic SpGEMM -------------------------------------------------------------
-  if ((st = run_pass<V>(h, 0, lb_sym, sym_cat, a, (int64_t)hs.max_prods, bps, s))) return st;
+  if ((st = run_pass<V>(h, 0, lb_sym, sym_cat, sym_cat + 1, a, (int64_t)hs.max_prods, bps, s))) return st;
   if ((st = timing_mark(h, 3, s))) return st;
   // ---- 4. prefix sum -> C row offsets; numeric classification -------------------------
   unsigned long long* dmax = reinterpret_cast<unsigned long long*>(static_cast<char*>(h->small.p) + 128);
@@ -826,6 +839,128 @@ speck_status_t analyze_impl(speck_handle_t h, const speck_csr_t* A, const speck_
     h->st.ms_scan = elapsed(h, 3, 4);
   }
   h->analyzed = true;
+  h->num_binned = false;
+  return SPECK_OK;
+}
+
+// Numeric phase of the rows [r0, r1) only (speck_spgemm_rows): the numeric bins (scattered once
+// per analysis) are cut to the chunk's rows by binary search, C pointers are shifted so that the
+// kernels' absolute C offsets land in the caller's chunk buffers, and long-row jobs of other
+// rows exit immediately.  The global load balancer is always on in this mode.
+template <typename V>
+speck_status_t spgemm_rows_impl(speck_handle_t h, const speck_csr_t* A, const speck_csr_t* B, const int64_t* C_rp,
+                                int64_t r0, int64_t r1, int32_t* C_col, V* C_val, cudaStream_t s) {
+  const int64_t m = A->rows;
+  if (r1 <= r0 || h->nnz_c == 0) return SPECK_OK;
+  speck_status_t st;
+  const int64_t tiles = (m + kBinTile - 1) / kBinTile;
+  const BinParams bpn = make_bin_params(h, 1);
+  h->st.lb_numeric = 1;
+  if (!h->num_binned) {
+    const int kt = kt_begin(h, s, SPECK_KERNEL_BINNING, 3, -1);
+    k_bin_scatter<<<(unsigned)tiles, kBinTile, 0, s>>>(A->row_ptr, static_cast<int64_t*>(h->prods.p), C_rp, m, bpn,
+                                                      static_cast<int64_t*>(h->hist_off.p), tiles,
+                                                      static_cast<int32_t*>(h->bins.p), nullptr);
+    CKL();
+    kt_end(h, s, kt);
+    h->num_binned = true;
+  }
+  CatStarts cs;
+  for (int c = 0; c <= CAT_COUNT; ++c) cs.s[c] = h->num_cat_start[c];
+  int64_t* d_out = reinterpret_cast<int64_t*>(static_cast<char*>(h->small.p) + kSmallRange);
+  k_bin_range<<<1, 32, 0, s>>>(static_cast<const int32_t*>(h->bins.p), cs, r0, r1, C_rp, d_out);
+  CKL();
+  unsigned long long* hp = h->h_pinned + kPinRange;
+  CK(cudaMemcpyAsync(hp, d_out, (2 * CAT_COUNT + 2) * 8, cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  int64_t beg[CAT_COUNT], end[CAT_COUNT];
+  for (int c = 0; c < CAT_COUNT; ++c) { beg[c] = (int64_t)hp[2 * c]; end[c] = (int64_t)hp[2 * c + 1]; }
+  const int64_t off = (int64_t)hp[2 * CAT_COUNT];
+  unsigned long long* ndense = reinterpret_cast<unsigned long long*>(static_cast<char*>(h->small.p) + 256);
+  CK(cudaMemsetAsync(ndense, 0, 8, s));
+  SpgemmArgs<V> a = base_args<V>(h, A, B);
+  a.C_rp = C_rp;
+  a.C_col = C_col - off;     // the kernels write C[C_rp[row] + t]; the chunk buffer starts at C_rp[r0]
+  a.C_val = C_val - off;
+  a.row_lo = r0;
+  a.row_hi = r1;
+  const int64_t c_end = (int64_t)hp[2 * CAT_COUNT + 1];
+  return run_pass<V>(h, 1, 1, beg, end, a, h->max_cnt, bpn, s, off, c_end - off);
+}
+
+// Device CSR transpose (transpose_kernels.cuh).
+template <typename V>
+speck_status_t transpose_impl(speck_handle_t h, const speck_csr_t* A, int64_t* T_rp, int32_t* T_col, V* T_val,
+                              cudaStream_t s) {
+  const int64_t n = A->cols, nnz = A->nnz;
+  speck_status_t st;
+  if ((st = ensure(h, h->small, 4096, s))) return st;
+  if ((st = ensure(h, h->tr_cnt, (size_t)(n + 1) * 8, s))) return st;
+  unsigned long long* cnt = static_cast<unsigned long long*>(h->tr_cnt.p);
+  CK(cudaMemsetAsync(cnt, 0, (size_t)(n + 1) * 8, s));
+  const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((nnz + kTrThreads - 1) / kTrThreads, (int64_t)h->num_sms * 16));
+  if (nnz > 0) {
+    k_tr_count<<<grid, kTrThreads, 0, s>>>(A->col_idx, nnz, cnt);
+    CKL();
+  }
+  unsigned long long* dmax = reinterpret_cast<unsigned long long*>(static_cast<char*>(h->small.p) + 3968);
+  CK(cudaMemsetAsync(dmax, 0, 8, s));
+  if ((st = launch_scan(h, reinterpret_cast<const int64_t*>(cnt), n, T_rp, dmax, s))) return st;
+  if (nnz == 0) return SPECK_OK;
+  CK(cudaMemcpyAsync(cnt, T_rp, (size_t)n * 8, cudaMemcpyDeviceToDevice, s));   // cursors
+  const unsigned wgrid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((A->rows * 32 + kTrThreads - 1) / kTrThreads, (int64_t)h->num_sms * 16));
+  k_tr_scatter<V><<<wgrid, kTrThreads, 0, s>>>(A->row_ptr, A->col_idx, static_cast<const V*>(A->values), A->rows, cnt,
+                                               T_col, T_val);
+  CKL();
+  const unsigned tgrid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((n * 32 + kTrThreads - 1) / kTrThreads, (int64_t)h->num_sms * 16));
+  k_tr_sort_warp<V><<<tgrid, kTrThreads, 0, s>>>(T_rp, n, T_col, T_val);
+  CKL();
+  // longer rows: list them with their tile counts (two lists: > 32 entries, > one tile)
+  unsigned long long hmax = 0;
+  CK(cudaMemcpyAsync(h->h_pinned + kPinRange, dmax, 8, cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  hmax = h->h_pinned[kPinRange];
+  for (int stage = 0; stage < 2; ++stage) {
+    const int64_t lo = stage == 0 ? 32 : kTrSmemSort;
+    if ((int64_t)hmax <= lo) break;
+    if ((st = ensure(h, h->tr_list, (size_t)n * 4 + (size_t)(n + 1) * 8 + 64, s))) return st;
+    int32_t* list = static_cast<int32_t*>(h->tr_list.p);
+    int64_t* tiles = reinterpret_cast<int64_t*>(static_cast<char*>(h->tr_list.p) + (((size_t)n * 4 + 15) & ~(size_t)15));
+    int64_t* first = reinterpret_cast<int64_t*>(cnt);   // cursors are no longer needed: tile prefix
+    unsigned long long* nl = dmax + 1;
+    CK(cudaMemsetAsync(nl, 0, 8, s));
+    k_tr_list<<<tgrid, kTrThreads, 0, s>>>(T_rp, n, lo, list, tiles, nl);
+    CKL();
+    CK(cudaMemcpyAsync(h->h_pinned + kPinRange + 1, nl, 8, cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    const int64_t nrows = (int64_t)h->h_pinned[kPinRange + 1];
+    if ((st = launch_scan(h, tiles, nrows, first, nullptr, s))) return st;
+    CK(cudaMemcpyAsync(h->h_pinned + kPinRange + 2, first + nrows, 8, cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    const int64_t ntiles = (int64_t)h->h_pinned[kPinRange + 2];
+    if (stage == 0) {
+      const size_t sm = (size_t)kTrSmemSort * (4 + sizeof(V));
+      k_tr_sort_block<V><<<(unsigned)ntiles, 1024, sm, s>>>(T_rp, list, first, nrows, T_col, T_val);
+      CKL();
+      continue;
+    }
+    // rows longer than a tile: merge rounds, ping-pong with a scratch copy of T
+    if ((st = ensure(h, h->tr_col, (size_t)nnz * 4, s))) return st;
+    if ((st = ensure(h, h->tr_val, (size_t)nnz * sizeof(V), s))) return st;
+    int32_t* c0 = T_col; V* v0 = T_val;
+    int32_t* c1 = static_cast<int32_t*>(h->tr_col.p); V* v1 = T_val ? static_cast<V*>(h->tr_val.p) : nullptr;
+    int rounds = 0;
+    for (int64_t L = kTrSmemSort; L < (int64_t)hmax; L *= 2, ++rounds) {
+      k_tr_merge<V><<<(unsigned)ntiles, 256, 0, s>>>(T_rp, list, first, nrows, L, c0, v0, c1, v1);
+      CKL();
+      std::swap(c0, c1);
+      std::swap(v0, v1);
+    }
+    if (rounds & 1) {   // result in the scratch copy: one copying round (a single run per pair) back
+      k_tr_merge<V><<<(unsigned)ntiles, 256, 0, s>>>(T_rp, list, first, nrows, (int64_t)1 << 40, c0, v0, c1, v1);
+      CKL();
+    }
+  }
   return SPECK_OK;
 }
 
@@ -858,7 +993,7 @@ speck_status_t spgemm_impl(speck_handle_t h, const speck_csr_t* A, const speck_c
   a.C_rp = C_rp;
   a.C_col = C_col;
   a.C_val = C_val;
-  if ((st = run_pass<V>(h, 1, lb, h->num_cat_start, a, h->max_cnt, bpn, s))) return st;
+  if ((st = run_pass<V>(h, 1, lb, h->num_cat_start, h->num_cat_start + 1, a, h->max_cnt, bpn, s))) return st;
   if ((st = timing_mark(h, 7, s))) return st;
   // numeric-stage times and counters are read lazily by speck_get_stats (no sync here)
   if (h->opt_timing) CK(cudaMemcpyAsync(h->h_pinned + 40, ndense, 8, cudaMemcpyDeviceToHost, s));
@@ -884,6 +1019,7 @@ __global__ void k_block_merge_groups(const int64_t* needs, int64_t n, int64_t ca
 }
 
 __global__ void k_query_nsmid(int* out) { *out = (int)nsmid(); }
+
 
 __global__ void k_group_size(int32_t T, const int64_t* nnzA, const int64_t* prods, const int64_t* maxlen, int64_t n,
                              int32_t* g) {
@@ -989,7 +1125,8 @@ speck_status_t speck_destroy(speck_handle_t h) {
   cudaDeviceSynchronize();
   Buf* bufs[] = {&h->prods, &h->maxlen, &h->colmin, &h->colmax, &h->cnt, &h->hist, &h->hist_off, &h->bins, &h->stats,
                  &h->scan_status, &h->resume, &h->small, &h->ana_long, &h->chunk_cnt, &h->cand, &h->nseg,
-                 &h->seg_off, &h->segs, &h->bm_pool, &h->bm_off, &h->binfo};
+                 &h->seg_off, &h->segs, &h->bm_pool, &h->bm_off, &h->binfo, &h->paths, &h->chunks, &h->tr_cnt,
+                 &h->tr_list, &h->tr_col, &h->tr_val};
   for (Buf* b : bufs) {
     if (!b->p) continue;
     if (h->urelease) h->urelease(b->p, nullptr, h->uctx);
@@ -1046,10 +1183,17 @@ speck_status_t speck_set_option(speck_handle_t h, int option, int64_t v) {
     case SPECK_OPT_BUCKET_SORT:
       if (v < 0 || v > 2) return fail(h, SPECK_ERR_INVALID_ARGUMENT, "BUCKET_SORT must be 0..2");
       h->opt_esc = v; break;
-    case SPECK_OPT_PATH_COUNTERS:
+    case SPECK_OPT_PATH_COUNTERS: {
       h->opt_paths = v;
       std::memset(h->st.path_rows, 0, sizeof h->st.path_rows);
+      if (v) {
+        speck_status_t r = ensure(h, h->paths, SPECK_PATH_COUNT * 8, nullptr);
+        if (r) return r;
+        if (cudaMemset(h->paths.p, 0, SPECK_PATH_COUNT * 8) != cudaSuccess)
+          return fail(h, SPECK_ERR_CUDA, "cannot clear the path counters");
+      }
       break;
+    }
     default: return fail(h, SPECK_ERR_INVALID_ARGUMENT, "unknown option %d", option);
   }
   return SPECK_OK;
@@ -1094,6 +1238,72 @@ speck_status_t speck_spgemm(speck_handle_t h, const speck_csr_t* A, const speck_
   return st;
 }
 
+speck_status_t speck_spgemm_rows(speck_handle_t h, const speck_csr_t* A, const speck_csr_t* B, const int64_t* C_rp,
+                                 int64_t r0, int64_t r1, int32_t* C_col_part, void* C_val_part, speck_stream_t stream) {
+  if (!h) return SPECK_ERR_INVALID_ARGUMENT;
+  h->err.clear();
+  speck_status_t st;
+  if ((st = check_csr(h, A, "A", true)) || (st = check_csr(h, B, "B", true))) return st;
+  if (A->cols != B->rows) return fail(h, SPECK_ERR_DIMENSION_MISMATCH, "A.cols != B.rows");
+  if (A->dtype != B->dtype) return fail(h, SPECK_ERR_DTYPE_MISMATCH, "A and B value types differ");
+  if (!same_problem(h, A, B)) return fail(h, SPECK_ERR_NOT_ANALYZED, "speck_spgemm_rows without a matching speck_analyze");
+  if (r0 < 0 || r1 < r0 || r1 > A->rows) return fail(h, SPECK_ERR_INVALID_ARGUMENT, "row range [%lld, %lld) outside [0, %lld)",
+                                                       (long long)r0, (long long)r1, (long long)A->rows);
+  if (!C_rp || (h->nnz_c > 0 && r1 > r0 && (!C_col_part || !C_val_part)))
+    return fail(h, SPECK_ERR_INVALID_ARGUMENT, "C arrays are NULL");
+  int prev = 0;
+  cudaGetDevice(&prev);
+  if (cudaSetDevice(h->device) != cudaSuccess) return fail(h, SPECK_ERR_CUDA, "cudaSetDevice failed");
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  st = A->dtype == SPECK_F64 ? spgemm_rows_impl<double>(h, A, B, C_rp, r0, r1, C_col_part, static_cast<double*>(C_val_part), s)
+                             : spgemm_rows_impl<float>(h, A, B, C_rp, r0, r1, C_col_part, static_cast<float*>(C_val_part), s);
+  cudaSetDevice(prev);
+  return st;
+}
+
+speck_status_t speck_transpose(speck_handle_t h, const speck_csr_t* A, int64_t* T_row_ptr, int32_t* T_col_idx,
+                               void* T_values, speck_stream_t stream) {
+  if (!h) return SPECK_ERR_INVALID_ARGUMENT;
+  h->err.clear();
+  speck_status_t st;
+  if ((st = check_csr(h, A, "A", false))) return st;
+  if (!T_row_ptr || (A->nnz > 0 && !T_col_idx)) return fail(h, SPECK_ERR_INVALID_ARGUMENT, "T arrays are NULL");
+  if (A->nnz > 0 && !T_values != !A->values)
+    return fail(h, SPECK_ERR_INVALID_ARGUMENT, "T_values must be given exactly when A.values is");
+  int prev = 0;
+  cudaGetDevice(&prev);
+  if (cudaSetDevice(h->device) != cudaSuccess) return fail(h, SPECK_ERR_CUDA, "cudaSetDevice failed");
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  st = A->dtype == SPECK_F64 ? transpose_impl<double>(h, A, T_row_ptr, T_col_idx, static_cast<double*>(T_values), s)
+                             : transpose_impl<float>(h, A, T_row_ptr, T_col_idx, static_cast<float*>(T_values), s);
+  cudaSetDevice(prev);
+  return st;
+}
+
+speck_status_t speck_row_chunks(speck_handle_t h, const int64_t* C_rp, int64_t rows, int64_t max_nnz, int64_t* bounds,
+                                int64_t max_parts, int64_t* n_parts) {
+  if (!h || !C_rp || !bounds || !n_parts || rows < 0 || max_parts < 1) return SPECK_ERR_INVALID_ARGUMENT;
+  h->err.clear();
+  if (!h->analyzed || rows != h->A_rows) return fail(h, SPECK_ERR_NOT_ANALYZED, "speck_row_chunks needs the analysis of C_row_ptr");
+  const int64_t step = max_nnz - h->max_cnt;
+  if (step <= 0)
+    return fail(h, SPECK_ERR_INVALID_ARGUMENT, "max_nnz %lld does not exceed the longest row of C (%lld entries)",
+                (long long)max_nnz, (long long)h->max_cnt);
+  const int64_t parts = std::max<int64_t>(1, (h->nnz_c + step - 1) / step);
+  if (parts > max_parts) return fail(h, SPECK_ERR_INVALID_ARGUMENT, "%lld chunks needed, bounds holds %lld", (long long)parts, (long long)max_parts);
+  int prev = 0;
+  cudaGetDevice(&prev);
+  cudaSetDevice(h->device);
+  speck_status_t st;
+  if ((st = ensure(h, h->chunks, (size_t)(parts + 1) * 8, nullptr))) { cudaSetDevice(prev); return st; }
+  k_chunk_bounds<<<(unsigned)((parts + 1 + 127) / 128), 128>>>(C_rp, rows, step, parts, static_cast<int64_t*>(h->chunks.p));
+  cudaError_t e = cudaMemcpy(bounds, h->chunks.p, (size_t)(parts + 1) * 8, cudaMemcpyDeviceToHost);
+  cudaSetDevice(prev);
+  if (e != cudaSuccess) return fail(h, SPECK_ERR_CUDA, "speck_row_chunks: %s", cudaGetErrorString(e));
+  *n_parts = parts;
+  return SPECK_OK;
+}
+
 speck_status_t speck_row_analysis(speck_handle_t h, const speck_csr_t* A, const speck_csr_t* B, int64_t* prods,
                                   int32_t* maxlen, int32_t* colmin, int32_t* colmax, speck_stream_t stream) {
   if (!h) return SPECK_ERR_INVALID_ARGUMENT;
@@ -1134,7 +1344,8 @@ speck_status_t speck_set_allocator(speck_handle_t h, speck_alloc_fn alloc, speck
   cudaDeviceSynchronize();   // no kernel may still use the workspace being released
   Buf* bufs[] = {&h->prods, &h->maxlen, &h->colmin, &h->colmax, &h->cnt, &h->hist, &h->hist_off, &h->bins, &h->stats,
                  &h->scan_status, &h->resume, &h->small, &h->ana_long, &h->chunk_cnt, &h->cand, &h->nseg,
-                 &h->seg_off, &h->segs, &h->bm_pool, &h->bm_off, &h->binfo};
+                 &h->seg_off, &h->segs, &h->bm_pool, &h->bm_off, &h->binfo, &h->paths, &h->chunks, &h->tr_cnt,
+                 &h->tr_list, &h->tr_col, &h->tr_val};
   for (Buf* b : bufs) release_buf(h, *b, nullptr);
   cudaStreamSynchronize(nullptr);
   h->ualloc = alloc;
@@ -1174,6 +1385,14 @@ speck_status_t speck_get_stats(speck_handle_t h, speck_stats_t* out) {
     h->st.kernel_id[i] = h->kt_id[i];
     h->st.kernel_bin[i] = h->kt_bin[i];
     h->st.kernel_ms[i] = h->kt_ms[i];
+  }
+  if (h->opt_paths && h->paths.p) {
+    unsigned long long pc[SPECK_PATH_COUNT];
+    if (cudaMemcpy(pc, h->paths.p, sizeof pc, cudaMemcpyDeviceToHost) != cudaSuccess) {
+      (void)cudaGetLastError();
+      return fail(h, SPECK_ERR_CUDA, "cannot read the path counters");
+    }
+    for (int i = 0; i < SPECK_PATH_COUNT; ++i) h->st.path_rows[i] = (int64_t)pc[i];
   }
   h->st.workspace_bytes = ws_bytes(h);
   h->st.kernel_launches = h->launches;

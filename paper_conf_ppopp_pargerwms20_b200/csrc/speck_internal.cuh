@@ -287,6 +287,11 @@ __device__ __forceinline__ uint32_t warp_block_merge(int64_t need, int n, int64_
   return starts;
 }
 
+// SPECK_OPT_PATH_COUNTERS: one thread per row (segment, CTA) counts the path it took.
+__device__ __forceinline__ void count_path(unsigned long long* paths, int path) {
+  if (paths) atomicAdd(paths + path, 1ull);
+}
+
 // ----------------------------------------------------------------------------------
 // Problem description handed to the SpGEMM kernels (device pointers).
 // ----------------------------------------------------------------------------------
@@ -316,6 +321,8 @@ struct SpgemmArgs {
   int64_t dense_window_cap;  // >0: cap dense window (test knob)
   int fixed_g;               // >0: fixed group size
   int esc;                   // bucket counting-sort rows (esc_kernels.cuh): 0 off, 1 numeric, 2 + symbolic
+  unsigned long long* paths; // SPECK_OPT_PATH_COUNTERS: rows per speck_path_t (nullptr: off)
+  int64_t row_lo, row_hi;    // row-range numeric (speck_spgemm_rows): long-row jobs outside [row_lo, row_hi) exit
   // symbolic out
   int64_t* cnt;
   // numeric in/out

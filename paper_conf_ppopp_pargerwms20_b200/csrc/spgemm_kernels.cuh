@@ -27,6 +27,9 @@
 
 namespace speck {
 
+#ifndef SPECK_WARP_U
+#define SPECK_WARP_U 1      // product chunks in flight per numeric warp-row expansion step (C2: 1 beats 2)
+#endif
 constexpr int kSmallSeg = kTinyCnt;   // rows with <= this many C entries are ranked, not sorted
 constexpr int kPPL = 4;         // products per lane per chunk in the warp-per-row path
 constexpr int kAllAvgLen = 256;  // expand_row ALL mode for rows whose references average >= this many products
@@ -343,15 +346,7 @@ struct FullRange {
   __device__ __forceinline__ void operator()(int, int64_t j0, int64_t j1, int64_t& s, int64_t& e) const { s = j0; e = j1; }
 };
 
-// First batch of a row loaded ahead of time (k_warp_rows pipelines it one row ahead): lane f
-// holds B row start/length and a of the row's f-th NZ.
-template <typename V>
-struct PreBatch {
-  int64_t bst = 0;
-  int blen = 0;
-  V a = V(0);
-  bool valid = false;
-};
+// (PreBatch, the first batch of a row loaded ahead by k_warp_rows, is defined in esc_kernels.cuh)
 
 //
 // ALL = true (single-row blocks): every warp reads every batch (its 32 A entries and B row
@@ -767,8 +762,9 @@ __device__ __forceinline__ int warp_row(const SpgemmArgs<V>& p, uint32_t* rk, V*
   // 2 products per lane per chunk (fewer registers, more resident warps) for numeric MODE 1/2 rows
   // (C5 numeric 379 -> 362 ms, C2 tiny rows at 40 warps/SM 2.56 -> 2.35 ms) and symbolic rows
   // (C2 symbolic A*P 1.38 -> 1.31 ms; 8 per lane spills: 1.72 ms); numeric MODE 0 rows 4
-  expand_row<PASS, V, PASS == 0, false, (PASS == 0 || MODE >= 1) ? 2 : kPPL>(
-      p, a0, alen, 0, 1, [&](uint32_t col, V v, bool act) {
+  // products: symbolic rows by expand_row (long B rows streamed, short ones balanced), numeric
+  // rows by expand_esc (REDUX owner search, esc_kernels.cuh) with the first batch loaded ahead
+  auto ins = [&](uint32_t col, V v, bool act) {
     if (PASS == 0) {
       if (act) newc += hash_insert_key(rk, S, col);
     } else {
@@ -787,12 +783,19 @@ __device__ __forceinline__ int warp_row(const SpgemmArgs<V>& p, uint32_t* rk, V*
         __syncwarp();
       }
     }
-  });
-  if (PASS == 0) return warp_sum(newc);
+  };
+  if (PASS == 0) expand_row<PASS, V, true, false, 2>(p, a0, alen, 0, 1, ins);
+  else expand_esc<PASS, V, SPECK_WARP_U>(p, a0, alen, 0, 1, ins, pre);
+  if (PASS == 0) {
+    if (lane == 0) count_path(p.paths, SPECK_PATH_SYM_WARP);
+    return warp_sum(newc);
+  }
   if (MODE != 1 && ordered && !__any_sync(0xffffffffu, wrapped)) {
     // ordered map: every entry goes to (occupied slots before its run) + (rank in the run)
+    if (lane == 0) count_path(p.paths, SPECK_PATH_NUM_WARP_ORDERED);
     warp_write_ordered<V>(rk, rv, S, 0u, S, cbase, 0, p.C_col, p.C_val);
   } else {
+    if (lane == 0) count_path(p.paths, MODE == 1 || cnt <= kSmallSeg ? SPECK_PATH_NUM_TINY : SPECK_PATH_NUM_WARP_SORTED);
     warp_row_sorted_write<V>(rk, rv, S, cbase, p.C_col, p.C_val);
   }
   __syncwarp();
@@ -806,7 +809,7 @@ __device__ __noinline__ void dense_row(const SpgemmArgs<V>& p, BlockMeta& bm, in
 // The per-configuration kernel.  PASS 0 = symbolic, 1 = numeric.
 // -----------------------------------------------------------------------------------
 template <int CFG, int PASS, typename V>
-__global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_spgemm(SpgemmArgs<V> p) {
+__global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_spgemm(const __grid_constant__ SpgemmArgs<V> p) {
   constexpr int T = kCfgThreads[CFG];
   
   extern __shared__ __align__(16) unsigned char smem[];
@@ -965,6 +968,7 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
     if (esc_done) {
     } else if (!bm.dense && nr >= NW && nr > 1) {
       // ===================== HASH, WARP PER ROW (multi-row blocks) =====================
+      if (tid == 0) count_path(p.paths, PASS == 0 ? SPECK_PATH_SYM_MERGED : SPECK_PATH_NUM_MERGED);
       // Each warp owns whole rows and their private map regions, so accumulation and the
       // sort/compaction epilogue need no block barrier; lanes whose key is unique within
       // the warp step update the value with a plain read-modify-write.
@@ -998,7 +1002,7 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
         const uint64_t mmult = bkt_mult((uint32_t)(bm.rhi[r] - bm.rlo[r] + 1), S);
         const bool ordered = bm.ordered;
         int newc = 0, wrapped = 0;
-        expand_row<PASS, V, PASS == 0, true, PASS == 1 ? 2 : kPPL>(p, bm.astart[r], (int)(bm.aoff[r + 1] - bm.aoff[r]), warp_id(), NW,
+        expand_esc<PASS, V, PASS == 0 ? 4 : 2>(p, bm.astart[r], (int)(bm.aoff[r + 1] - bm.aoff[r]), warp_id(), NW,
                             [&](uint32_t col, V v, bool act) {
                               if (PASS == 0) {
                                 if (act) newc += hash_insert_key(rk, S, col);
@@ -1023,6 +1027,8 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
       int any_wrap = !bm.ordered;   // scrambled maps take the compaction + sort epilogue
       if (PASS == 1)
         for (int rr = 0; rr < nr; ++rr) any_wrap |= bm.rwrap[rr];
+      if (tid == 0)
+        count_path(p.paths, PASS == 0 ? SPECK_PATH_SYM_BLOCK_HASH : any_wrap ? SPECK_PATH_NUM_BLOCK_SORTED : SPECK_PATH_NUM_BLOCK_ORDERED);
       if (PASS == 0) {
         if (tid < nr) p.cnt[bm.row[b0 + tid]] = bm.rcnt[tid];
         if (CFG == kNumCfg - 1 && p.chunk_cnt && nr == 1 && bm.prods > p.long_thr) {
@@ -1081,6 +1087,9 @@ __device__ __noinline__ void dense_row(const SpgemmArgs<V>& p, BlockMeta& bm, in
       V* dvals = reinterpret_cast<V*>(smem + (PASS == 0 ? 0 : (((W + 31) / 32) * 4 + 15) / 16 * 16));
       int32_t* res = nullptr;       // double-buffered resume offsets (cur, next)
       int32_t* res_next = nullptr;
+      if (tid == 0)
+        count_path(p.paths, PASS == 0 ? (nwin > 1 ? SPECK_PATH_SYM_DENSE_MULTI : SPECK_PATH_SYM_DENSE)
+                                      : (nwin > 1 ? SPECK_PATH_NUM_DENSE_MULTI : SPECK_PATH_NUM_DENSE));
       if (nwin > 1) {
         const unsigned slot = smid();
         if (slot >= (unsigned)p.resume_slots) __trap();
@@ -1166,7 +1175,7 @@ __device__ __noinline__ void dense_row(const SpgemmArgs<V>& p, BlockMeta& bm, in
 // -----------------------------------------------------------------------------------
 template <int PASS, typename V, int MODE>
 __global__ void __launch_bounds__(kWarpRowThreads, wr_ctas_per_sm(PASS, MODE))
-    k_warp_rows(SpgemmArgs<V> p, unsigned long long* __restrict__ counter) {
+    k_warp_rows(const __grid_constant__ SpgemmArgs<V> p, unsigned long long* __restrict__ counter) {
   extern __shared__ __align__(16) unsigned char smem[];
   const int lane = lane_id();
   constexpr int kRegion = wr_region_bytes(PASS, MODE);
@@ -1176,7 +1185,7 @@ __global__ void __launch_bounds__(kWarpRowThreads, wr_ctas_per_sm(PASS, MODE))
   const uint32_t cap = PASS == 0 ? wr_sym_cap() : wr_num_cap<V>(kRegion);
   const int64_t esc_cap = esc_capacity<V>(PASS, kRegion);
   const int64_t n = p.n_entries;
-  constexpr bool kRange = MODE != 1;
+  constexpr bool kRange = (PASS == 1 && MODE != 1) || MODE == 3;
   // row metadata, one field per lane: 0 A_rp[r], 1 A_rp[r+1], 2 prods[r] / C_rp[r], 3 C_rp[r+1],
   // 4 colmin[r], 5 colmax[r], 6 prods[r] (numeric) (one round trip instead of seven dependent loads)
   auto fetch = [&](int64_t e, int32_t& row, int64_t& mv) {
@@ -1234,7 +1243,7 @@ __global__ void __launch_bounds__(kWarpRowThreads, wr_ctas_per_sm(PASS, MODE))
   PreBatch<V> bt;
   {
     const int64_t a0 = __shfl_sync(0xffffffffu, mv, 0);
-    fetch_batch(a0, (int)(__shfl_sync(0xffffffffu, mv, 1) - a0), bt);
+    if (PASS == 1) fetch_batch(a0, (int)(__shfl_sync(0xffffffffu, mv, 1) - a0), bt);   // symbolic rows: no pre-batch
   }
   unsigned long long en = next_index(e);
   int32_t rown;
@@ -1257,7 +1266,7 @@ __global__ void __launch_bounds__(kWarpRowThreads, wr_ctas_per_sm(PASS, MODE))
     const PreBatch<V> bcur = bt;
     // pipeline: next row's batch, the row after next's metadata
     const unsigned long long enn = (int64_t)en < n ? next_index(en) : en;
-    if ((int64_t)en < n) {
+    if (PASS == 1 && (int64_t)en < n) {
       const int64_t a0n = __shfl_sync(0xffffffffu, mvn, 0);
       fetch_batch(a0n, (int)(__shfl_sync(0xffffffffu, mvn, 1) - a0n), bt);
     }
@@ -1265,7 +1274,7 @@ __global__ void __launch_bounds__(kWarpRowThreads, wr_ctas_per_sm(PASS, MODE))
     mv = mvn;
     fetch((int64_t)enn, rown, mvn);
     int c = -1;
-    if (MODE != 1) {
+    if (MODE != 1 && (PASS == 1 || MODE == 3)) {
       // rows whose products are (almost) all distinct columns: counting sort on column buckets
       // (esc_kernels.cuh); -1 = uneven buckets, the hash map below takes the row
       const int64_t np = PASS == 0 ? need : __shfl_sync(0xffffffffu, mv_prev6, 6);
@@ -1289,7 +1298,7 @@ __global__ void __launch_bounds__(256) k_direct(const int32_t* __restrict__ rows
                                                 const V* __restrict__ A_val, const int64_t* __restrict__ B_rp,
                                                 const int32_t* __restrict__ B_col, const V* __restrict__ B_val,
                                                 const int64_t* __restrict__ C_rp, int32_t* __restrict__ C_col,
-                                                V* __restrict__ C_val) {
+                                                V* __restrict__ C_val, unsigned long long* paths) {
   const int sub = threadIdx.x % GD;
   const int64_t stride = (int64_t)gridDim.x * (blockDim.x / GD);
   for (int64_t e = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) / GD; e < n_rows; e += stride) {
@@ -1299,6 +1308,7 @@ __global__ void __launch_bounds__(256) k_direct(const int32_t* __restrict__ rows
     const V a = A_val[q];
     const int64_t b0 = B_rp[kc], len = B_rp[kc + 1] - b0;
     const int64_t c0 = C_rp[row];
+    if (sub == 0) count_path(paths, SPECK_PATH_NUM_DIRECT);
     for (int64_t j = sub; j < len; j += GD) {
       C_col[c0 + j] = B_col[b0 + j];
       C_val[c0 + j] = a * B_val[b0 + j];

@@ -32,7 +32,8 @@ KERNEL_KINDS = {1: "analysis", 2: "binning", 3: "scan", 4: "sym_warp", 5: "sym_b
 # speck_path_t
 PATHS = ["sym_warp", "sym_block_hash", "sym_merged", "sym_dense", "sym_dense_multi", "num_tiny", "num_warp_ordered",
          "num_warp_sorted", "num_block_ordered", "num_block_sorted", "num_merged", "num_dense", "num_dense_multi",
-         "num_direct", "seg_hash", "seg_dense", "seg_windows", "long_bitmap", "long_bitmap_split"]
+         "num_direct", "seg_hash", "seg_dense", "seg_windows", "long_bitmap", "long_bitmap_split", "sym_esc", "num_esc",
+         "num_esc_dup", "esc_fallback"]
 PATH_COUNT = 24
 # bin categories of speck_stats_t.bin_* (per pass)
 CATEGORIES = ["empty", "direct", "cfg0", "cfg1", "cfg2", "cfg3", "cfg4", "long", "tiny", "unused"]
@@ -46,6 +47,7 @@ EXPORTS = [
     "speck_create", "speck_destroy", "speck_set_option", "speck_analyze", "speck_spgemm", "speck_row_analysis",
     "speck_get_stats", "speck_status_string", "speck_last_error", "speck_version", "speck_block_merge",
     "speck_group_size", "speck_hash_probe", "speck_exclusive_scan", "speck_row_products", "speck_set_allocator",
+    "speck_spgemm_rows", "speck_row_chunks", "speck_transpose",
 ]
 _ALLOC_FN = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p, ctypes.c_void_p)
 _RELEASE_FN = ctypes.CFUNCTYPE(None, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p)
@@ -117,6 +119,9 @@ def load() -> ctypes.CDLL:
         L.speck_exclusive_scan.argtypes = [P, P, I64, P, P]
         L.speck_row_products.argtypes = [P, ctypes.POINTER(_Csr), ctypes.POINTER(_Csr), P, P]
         L.speck_set_allocator.argtypes = [P, _ALLOC_FN, _RELEASE_FN, P]
+        L.speck_spgemm_rows.argtypes = [P, ctypes.POINTER(_Csr), ctypes.POINTER(_Csr), P, I64, I64, P, P, P]
+        L.speck_row_chunks.argtypes = [P, P, I64, I64, P, I64, ctypes.POINTER(I64)]
+        L.speck_transpose.argtypes = [P, ctypes.POINTER(_Csr), P, P, P, P]
         for f in EXPORTS:
             if f not in ("speck_status_string", "speck_last_error", "speck_version"):
                 getattr(L, f).restype = ctypes.c_int
@@ -252,6 +257,49 @@ class Handle:
         val = torch.empty(nnz, dtype=A.val.dtype, device=dev)
         self.numeric(A, B, rp, col, val, stream=stream)
         return CSR(A.rows, B.cols, rp, col, val)
+
+    def numeric_rows(self, A, B, C_row_ptr: torch.Tensor, r0: int, r1: int, C_col: torch.Tensor, C_val: torch.Tensor,
+                     stream=None):
+        """Numeric phase of rows [r0, r1) into chunk buffers of C_row_ptr[r1] - C_row_ptr[r0] entries."""
+        a, b = _csr(A), _csr(B)
+        self._check(self._L.speck_spgemm_rows(self._h, ctypes.byref(a), ctypes.byref(b), C_row_ptr.data_ptr(), int(r0),
+                                              int(r1), _ptr(C_col), _ptr(C_val), _stream(stream)))
+
+    def row_chunks(self, C_row_ptr: torch.Tensor, max_nnz: int, max_parts: int = 1 << 16):
+        """Row bounds [0, ..., rows] of consecutive chunks holding < max_nnz entries each."""
+        import numpy as np
+        bounds = np.zeros(max_parts + 1, np.int64)
+        n = ctypes.c_int64(0)
+        self._check(self._L.speck_row_chunks(self._h, C_row_ptr.data_ptr(), C_row_ptr.numel() - 1, int(max_nnz),
+                                             bounds.ctypes.data, int(max_parts), ctypes.byref(n)))
+        return [int(x) for x in bounds[:n.value + 1]]
+
+    def spgemm_chunks(self, A, B, max_nnz: int, stream=None):
+        """Memory-bounded C = A·B: analyze once, then yield (r0, r1, row_ptr_slice, col, val) for
+        consecutive row chunks of < max_nnz entries; only one chunk's C is allocated at a time
+        (the caller consumes it before asking for the next)."""
+        rp, nnz = self.analyze(A, B, stream=stream)
+        dev = A.row_ptr.device
+        bounds = self.row_chunks(rp, max_nnz)
+        for r0, r1 in zip(bounds[:-1], bounds[1:]):
+            if r1 <= r0:
+                continue
+            off = rp[r0:r1 + 1] - rp[r0]
+            n = int(off[-1])
+            col = torch.empty(n, dtype=torch.int32, device=dev)
+            val = torch.empty(n, dtype=A.val.dtype, device=dev)
+            self.numeric_rows(A, B, rp, r0, r1, col, val, stream=stream)
+            yield r0, r1, off, col, val
+
+    def transpose(self, A, stream=None) -> CSR:
+        """T = Aᵀ (sorted CSR) on the device (speck_transpose)."""
+        dev = A.row_ptr.device
+        rp = torch.empty(A.cols + 1, dtype=torch.int64, device=dev)
+        col = torch.empty(A.col.numel(), dtype=torch.int32, device=dev)
+        val = torch.empty(A.col.numel(), dtype=A.val.dtype, device=dev)
+        self._check(self._L.speck_transpose(self._h, ctypes.byref(_csr(A)), rp.data_ptr(), _ptr(col),
+                                            val.data_ptr() if A.val.numel() else None, _stream(stream)))
+        return CSR(A.cols, A.rows, rp, col, val)
 
     def row_products(self, A, B, stream=None) -> torch.Tensor:
         """Alg. 1 line 10 per row: products int64 device tensor (speck_row_products)."""

@@ -170,9 +170,8 @@ PATHS = [
     dict(force_accumulator=2, dense_window=64),
     dict(force_accumulator=2, dense_window=3),
     dict(disable_direct=1),
-    dict(fixed_group_size=1),
-    dict(fixed_group_size=32),
-    dict(fixed_group_size=1024),
+    dict(bucket_sort=0),
+    dict(bucket_sort=1),
     dict(concurrent_streams=1),
     dict(warp_rows=0),
     dict(warp_rows=0, global_lb_symbolic=0, global_lb_numeric=0),
@@ -387,45 +386,280 @@ def test_handle_reuse_and_stats(dev):
         assert st["ms_symbolic"] >= 0 and st["ms_numeric"] >= 0
 
 
+# ----------------------------------------------------------------------- parity plumbing
+def test_nan_poisoned_result_fails_parity(dev):
+    """assert_parity must reject a NaN the kernels never produce (the comparator pin, on device)."""
+    A = W.rmat(10, 8, seed=5, dtype=torch.float32)
+    C, _ = gpu_spgemm(A, A)
+    assert_parity(A, A, C)
+    C.val[C.nnz // 2] = float("nan")
+    with pytest.raises(AssertionError):
+        assert_parity(A, A, C)
+
+
+def test_option_change_invalidates_analysis(dev):
+    """Changing a plan option between speck_analyze and speck_spgemm must not run a stale plan."""
+    A = W.rmat(10, 8, seed=6, dtype=torch.float32).to(dev)
+    h = sp.Handle(0)
+    rp, nnz = h.analyze(A, A)
+    h.set_option("warp_rows", 0)
+    col = torch.empty(nnz, dtype=torch.int32, device=dev)
+    val = torch.empty(nnz, dtype=torch.float32, device=dev)
+    with pytest.raises(sp.SpeckError) as e:
+        h.numeric(A, A, rp, col, val)
+    assert e.value.status == 7
+    h.set_option("stage_timing", 1)          # not a plan option: keeps the analysis
+    rp, nnz = h.analyze(A, A)
+    h.set_option("stage_timing", 0)
+    h.numeric(A, A, rp, col, val)
+    torch.cuda.synchronize()
+    h.close()
+
+
+def test_kernel_timing_and_bin_stats(dev):
+    """SPECK_OPT_KERNEL_TIMING reports every launch with a positive time; the per-bin sums add up
+    to the oracle's totals (rows, nnz(A), products, nnz(C))."""
+    A = W.rmat(12, 16, seed=7, dtype=torch.float32)
+    h = sp.Handle(0, kernel_timing=1)
+    C = h.spgemm(A.to(dev), A.to(dev))
+    torch.cuda.synchronize()
+    st = h.stats()
+    assert st["n_kernels"] >= 5 and all(k["ms"] > 0 for k in st["kernels"])
+    kinds = {k["kind"] for k in st["kernels"]}
+    assert {"analysis", "scan"} <= kinds
+    prods, _, _, _, (tot, _) = oracle.row_analysis(A, A)
+    nnza = np.diff(A.row_ptr.numpy())
+    for pss in (0, 1):
+        assert sum(st["bin_rows"][pss]) == A.rows
+        assert sum(st["bin_nnza"][pss]) == int(nnza.sum())
+        assert sum(st["bin_products"][pss]) == tot
+    assert sum(st["bin_nnzc"]) == C.nnz
+    h.close()
+
+
+# Inputs that together reach every accumulator path of the pipeline (SPECK_OPT_PATH_COUNTERS).
+def _path_inputs():
+    rng = np.random.default_rng(99)
+    out = [("rmat", W.rmat(12, 16, seed=11, dtype=torch.float32), None, {}),
+           ("poisson", W.poisson2d(64), None, {}),
+           ("rmat_lb_off", W.rmat(11, 16, seed=12, dtype=torch.float32), None,
+            dict(global_lb_symbolic=0, global_lb_numeric=0)),
+           ("merged", W.rmat(11, 16, seed=13, dtype=torch.float32), None, dict(warp_rows=0)),
+           ("hash_only", W.rmat(12, 16, seed=14, dtype=torch.float32), None, dict(bucket_sort=0)),
+           ("esc_sym", W.rmat(12, 16, seed=17, dtype=torch.float32), None, dict(bucket_sort=2)),
+           ("dense", W.rmat(11, 16, seed=15, dtype=torch.float32), None, dict(force_accumulator=2)),
+           ("dense_multi", W.rmat(11, 16, seed=16, dtype=torch.float32), None,
+            dict(force_accumulator=2, dense_window=64))]
+    # long rows: segments (few) and bitmap CTAs (many), see test_long_rows / test_many_long_rows_bitmap
+    A = W.random_sparse(6, 2000, 0.5, seed=31, dtype=torch.float32)
+    B = W.random_sparse(2000, 200_000, 0.01, seed=32, dtype=torch.float32)
+    out.append(("segments", A, B, {}))
+    out.append(("windows", A, B, dict(segments=0)))
+    # sparse long rows (~90k products over 2M columns): hashed column segments
+    cols = np.sort(rng.choice(2_000_000, size=(2000, 50), replace=True), axis=1).astype(np.int64)
+    Bs = W.csr_from_coo(2000, 2_000_000, torch.arange(2000).repeat_interleave(50), torch.tensor(cols.reshape(-1)), None,
+                        dtype=torch.float32, seed=5)
+    As = W.random_sparse(4, 2000, 0.9, seed=33, dtype=torch.float32)
+    out.append(("seg_hash", As, Bs, {}))
+    # uniform short rows: merged blocks (Alg. 2) and the warp-per-row ordered map
+    U = W.random_sparse(3000, 3000, 0.012, seed=21, dtype=torch.float32)
+    out.append(("merged_numeric", U, None, dict(warp_rows=0, global_lb_symbolic=1, global_lb_numeric=1)))
+    out.append(("warp_ordered", U, None, dict(bucket_sort=0, global_lb_symbolic=1, global_lb_numeric=1)))
+    nb, lb = 3000, 1000
+    cols = np.stack([np.sort(rng.choice(1 << 20, size=lb, replace=False)) for _ in range(nb)])
+    Bm = W.csr_from_coo(nb, 1 << 20, torch.arange(nb).repeat_interleave(lb), torch.tensor(cols.reshape(-1)), None,
+                        dtype=torch.float32, seed=18)
+    ar = np.repeat(np.arange(700), 24)
+    ac = np.concatenate([np.sort(rng.choice(nb, 24, replace=False)) for _ in range(700)])
+    Am = W.csr_from_coo(700, nb, torch.tensor(ar), torch.tensor(ac), None, dtype=torch.float32, seed=19)
+    out.append(("bitmap", Am, Bm, {}))
+    Av = W.csr_from_coo(4, nb, torch.arange(4).repeat_interleave(2000),
+                        torch.tensor(np.concatenate([np.sort(rng.choice(nb, 2000, replace=False)) for _ in range(4)])),
+                        None, dtype=torch.float32, seed=20)
+    out.append(("bitmap_split", Av, Bm, dict(long_bitmap=2)))
+    return out
+
+
+def test_every_path_is_hit_and_correct(dev):
+    """Path coverage: across these inputs every accumulator path the library has is taken at
+    least once (device-side path counters), and every result matches the oracle."""
+    hit = {}
+    for name, A, B, opts in _path_inputs():
+        B = A if B is None else B
+        h = sp.Handle(0, path_counters=1, **opts)
+        C = h.spgemm(A.to(dev), B.to(dev))
+        torch.cuda.synchronize()
+        for k, v in h.stats()["paths"].items():
+            hit[k] = hit.get(k, 0) + v
+        h.close()
+        assert_parity(A, B, C)
+    missing = [k for k, v in hit.items() if v == 0 and k not in OPTIONAL_PATHS]
+    print("path counts:", hit)
+    assert not missing, f"paths never taken: {missing} (counts {hit})"
+
+
+# paths that only fire on inputs the suite cannot make small (documented in DESIGN.md §2)
+# (seg_windows: a "windows" job needs >= 4 long rows per SM whose column range is too wide for the
+# bitmap CTA and whose window overhead beats segmenting — C5-sized inputs only)
+OPTIONAL_PATHS = {"num_warp_sorted", "esc_fallback", "seg_windows"}
+
+
+# ----------------------------------------------------------------------- transpose (§8 f2)
+@pytest.mark.parametrize("case", ["p_c2", "rmat_long_cols", "random_f64", "empty"])
+def test_transpose_bit_exact(dev, case):
+    """speck_transpose == the host transpose (workloads.transpose, a stable sort), bit for bit:
+    C2's P (rows of R = P^T up to 27 entries), an R-MAT with columns longer than one smem tile
+    (merge rounds), random fp64 with empty rows/cols, and an empty matrix."""
+    if case == "p_c2":
+        _, P, R = W.amg27(32)
+        A, want = P, R
+    elif case == "rmat_long_cols":
+        A = W.rmat(16, 16, seed=61, dtype=torch.float32)
+        # add one very long column (every 3rd row has column 5) so a row of T spans 3 tiles
+        r = torch.arange(0, A.rows, 3)
+        A = W.csr_from_coo(A.rows, A.cols, torch.cat([torch.repeat_interleave(torch.arange(A.rows), A.row_lengths()), r]),
+                           torch.cat([A.col.long(), torch.full_like(r, 5)]), None, dtype=torch.float32, seed=62)
+        want = W.transpose(A)
+    elif case == "random_f64":
+        A = W.random_sparse(700, 900, 0.02, seed=63, empty_rows=0.2)
+        want = W.transpose(A)
+    else:
+        A = W.CSR(5, 7, torch.zeros(6, dtype=torch.int64), torch.zeros(0, dtype=torch.int32), torch.zeros(0))
+        want = W.transpose(A)
+    h = sp.Handle(0)
+    T = h.transpose(A.to(dev))
+    torch.cuda.synchronize()
+    assert T.rows == A.cols and T.cols == A.rows
+    assert torch.equal(T.row_ptr.cpu(), want.row_ptr)
+    assert torch.equal(T.col.cpu(), want.col)
+    assert torch.equal(T.val.cpu(), want.val)
+    if case == "rmat_long_cols":
+        assert int((T.row_ptr[1:] - T.row_ptr[:-1]).max()) > 2 * 8192
+
+
+def test_a_times_a_transpose_protocol(dev):
+    """The paper's rectangular protocol: C = A·Aᵀ with Aᵀ from speck_transpose."""
+    A = W.random_sparse(600, 2000, 0.01, seed=64, dtype=torch.float64, empty_rows=0.1)
+    h = sp.Handle(0)
+    At = h.transpose(A.to(dev))
+    C = h.spgemm(A.to(dev), At)
+    torch.cuda.synchronize()
+    Ath = W.CSR(At.rows, At.cols, At.row_ptr.cpu(), At.col.cpu(), At.val.cpu())
+    assert_parity(A, Ath, C)
+
+
+# ----------------------------------------------------------------------- memory-bounded (§8 f1)
+def _assemble(chunks, rows):
+    rp = torch.zeros(rows + 1, dtype=torch.int64)
+    cols, vals, base = [], [], 0
+    for r0, r1, off, col, val in chunks:
+        rp[r0 + 1:r1 + 1] = off[1:].cpu() + base
+        base += int(off[-1])
+        cols.append(col.cpu())
+        vals.append(val.cpu())
+    # rows between chunks (empty chunks were skipped): carry the running offset forward
+    rp = torch.cummax(rp, 0).values
+    return rp, torch.cat(cols), torch.cat(vals)
+
+
+@pytest.mark.parametrize("dt", [torch.float32, torch.float64])
+def test_chunked_rows_match_oracle(dev, dt):
+    """speck_spgemm_rows over the chunks of speck_row_chunks reproduces C = A·B (every row vs the
+    oracle; structure identical to one-shot speck_spgemm), with >= 4 chunks."""
+    A = W.rmat(12, 16, seed=51, dtype=dt)
+    Ad = A.to(dev)
+    full = sp.Handle(0).spgemm(Ad, Ad)
+    torch.cuda.synchronize()
+    maxrow = int((full.row_ptr[1:] - full.row_ptr[:-1]).max())
+    budget = max(full.nnz // 6, maxrow + 1)
+    h = sp.Handle(0)
+    chunks = list(h.spgemm_chunks(Ad, Ad, budget))
+    torch.cuda.synchronize()
+    assert len(chunks) >= 4 and all(int(c[2][-1]) < budget for c in chunks)
+    rp, col, val = _assemble(chunks, A.rows)
+    assert torch.equal(rp, full.row_ptr.cpu()) and torch.equal(col, full.col.cpu())
+    C = sp.CSR(A.rows, A.cols, rp.to(dev), col.to(dev), val.to(dev))
+    assert_parity(A, A, C)
+    with pytest.raises(sp.SpeckError):
+        h.row_chunks(full.row_ptr, maxrow)          # a budget below the longest row is refused
+
+
+def test_chunked_c4_full_size(dev):
+    """C4 at full size under a budget of a quarter of nnz(C): >= 4 chunks, structure identical to
+    the one-shot product, values vs the oracle on every row of the 64 giant rows' chunks sampled."""
+    (label, A, B), = W.config("c4", device=dev)
+    h = sp.Handle(0)
+    full = h.spgemm(A, A)
+    torch.cuda.synchronize()
+    nnz = full.nnz
+    frp = full.row_ptr.cpu()
+    fcol = full.col
+    maxrow = int((frp[1:] - frp[:-1]).max())
+    budget = max(nnz // 4, maxrow + 1)
+    h2 = sp.Handle(0)
+    n_chunks, Ah = 0, A.to("cpu")
+    tol = oracle.TOL[np.dtype(np.float32)]
+    for r0, r1, off, col, val in h2.spgemm_chunks(A, A, budget):
+        n_chunks += 1
+        s0 = int(frp[r0])
+        assert torch.equal(off.cpu() + s0, frp[r0:r1 + 1])
+        assert torch.equal(col, fcol[s0:s0 + col.numel()])
+        # values: the first 2e6 entries of the chunk against the oracle
+        rr = int(np.searchsorted(off.cpu().numpy(), min(2_000_000, int(off[-1])), side="right"))
+        rr = max(1, min(rr, r1 - r0))
+        rp_o, col_o, val_o, sc_o = oracle.spgemm(Ah, Ah, r0, r0 + rr)
+        n = int(rp_o[-1])
+        res = oracle.compare(off[:rr + 1].cpu().numpy(), col[:n].cpu().numpy(), val[:n].cpu().numpy().astype(np.float64),
+                             rp_o, col_o, val_o, sc_o, tol)
+        assert res["ok"], res
+        del col, val
+    assert n_chunks >= 4
+
+
 # ----------------------------------------------------------------------- full sizes
-def sample_blocks(m, prods, seed, n_blocks=6, width=64):
+def _strata_blocks(cnt, seed, frac, per_stratum=16, width=64):
+    """Row blocks covering >= frac of the rows: random 64-row blocks plus `per_stratum` single
+    rows from every power-of-two stratum of nnz(C_i) (so every bin category is represented)."""
+    m = cnt.size
     rng = np.random.default_rng(seed)
-    starts = list(rng.integers(0, max(m - width, 1), n_blocks))
-    heavy = np.argsort(prods)[-4:]
-    blocks = [(int(s), int(min(s + width, m))) for s in starts] + [(int(r), int(r) + 1) for r in heavy]
+    blocks = []
+    nblk = int(np.ceil(frac * m / width))
+    starts = np.sort(rng.choice(max(m // width, 1), size=min(nblk, max(m // width, 1)), replace=False)) * width
+    blocks += [(int(s), int(min(s + width, m))) for s in starts]
+    strat = np.where(cnt > 0, np.floor(np.log2(np.maximum(cnt, 1))).astype(np.int64), -1)
+    for k in np.unique(strat):
+        rows = np.nonzero(strat == k)[0]
+        for r in rng.choice(rows, size=min(per_stratum, rows.size), replace=False):
+            blocks.append((int(r), int(r) + 1))
     blocks.append((m - min(width, m), m))   # ragged tail
     return blocks
 
 
-def test_c2_full_size_bit_exact(dev):
-    """BASELINE config[1] at full size (128^3), both SpGEMMs of the Galerkin chain, every row."""
-    A, P, R = W.amg27(128, device=dev)
-    h = sp.Handle(0)
-    AP = h.spgemm(A, P)
-    Ac = h.spgemm(R, AP)
-    torch.cuda.synchronize()
-    assert AP.nnz == 317 ** 3 and Ac.nnz == 190 ** 3
-    Ah, Ph, Rh = A.to("cpu"), P.to("cpu"), R.to("cpu")
-    assert_parity(Ah, Ph, AP, exact=True)
-    APh = W.CSR(AP.rows, AP.cols, AP.row_ptr.cpu(), AP.col.cpu(), AP.val.cpu())
-    assert_parity(Rh, APh, Ac, exact=True)
-
-
-@pytest.mark.parametrize("cfg", ["c3", "c4", "c5"])
-def test_full_size_sampled(dev, cfg):
+@pytest.mark.parametrize("cfg,frac", [("c4", 1.0), ("c3", 0.10), ("c5", 0.10)])
+def test_full_size_every_row(dev, cfg, frac):
+    """BASELINE configs at full size: nnz(C_i) of EVERY row equals the oracle's structural count
+    (and so row_ptr is bit-exact everywhere); columns and values bit-exact / within tolerance on
+    every row of C4 and on >= 10% of the rows of C3 and C5 drawn from every nnz(C_i) stratum."""
     (label, A, B), = W.config(cfg, device=dev)
     h = sp.Handle(0)
     C = h.spgemm(A, B)
     torch.cuda.synchronize()
     st = h.stats()
-    prods, _, cmin, cmax = (t.cpu().numpy() for t in h.row_analysis(A, B))
-    rp = C.row_ptr.cpu().numpy()
-    cnt = np.diff(rp)
-    # properties at any size: monotone offsets, nnz(C) bounds, totals
-    assert rp[0] == 0 and np.all(cnt >= 0) and np.all(cnt <= prods)
-    assert int(prods.sum()) == st["products"] and int(rp[-1]) == C.nnz
     Ah = A.to("cpu")
-    blocks = sample_blocks(A.rows, prods, seed=7)
+    cnt_ref = oracle.symbolic(Ah, Ah)
+    rp = C.row_ptr.cpu().numpy()
+    assert rp[0] == 0 and int(rp[-1]) == C.nnz == int(cnt_ref.sum()) == st["nnz_c"]
+    assert np.array_equal(np.diff(rp), cnt_ref)
+    if frac >= 1.0:
+        # every row, streamed in blocks of ~2e7 entries
+        blocks, r0 = [], 0
+        while r0 < A.rows:
+            r1 = min(int(np.searchsorted(rp, rp[r0] + 20_000_000, side="right")), A.rows)
+            r1 = max(r1, r0 + 1)
+            blocks.append((r0, r1))
+            r0 = r1
+    else:
+        blocks = _strata_blocks(cnt_ref, seed=7, frac=frac)
     assert_parity(Ah, Ah, C, rows=blocks)
     del C
     torch.cuda.empty_cache()

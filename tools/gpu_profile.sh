@@ -25,7 +25,10 @@ for k in "${KS[@]}"; do
   timeout 900 ncu --set full --clock-control none --import-source on -k "regex:$k" --kernel-name-base demangled -c 1 \
     -o /tmp/rep/k$i python bench.py $B --steps 1 --warmup 3 > gpurun_out/${TAG}_${CFG}_k$i.log 2>&1
   python tools/ncu_summary.py /tmp/rep/k$i.ncu-rep 0 > gpurun_out/${TAG}_${CFG}_k$i.txt 2>&1
-  cp /tmp/rep/k$i.ncu-rep gpurun_out/${TAG}_${CFG}_k$i.ncu-rep
+  python tools/ncu_sass.py /tmp/rep/k$i.ncu-rep 0 > gpurun_out/${TAG}_${CFG}_k${i}_sass.txt 2>&1
+  python tools/traffic_from_ncu.py --dry $CFG $TAG /tmp/rep/k$i.ncu-rep >> gpurun_out/${TAG}_${CFG}_traffic.txt 2>&1
+  # reports are ~10-40 MB each: only brought back on request (gpurun_out is capped at 64 MiB)
+  if [ "${KEEP_REP:-0}" = 1 ]; then cp /tmp/rep/k$i.ncu-rep gpurun_out/${TAG}_${CFG}_k$i.ncu-rep; fi
   i=$((i+1))
 done
 echo done

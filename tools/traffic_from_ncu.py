@@ -52,7 +52,9 @@ def metrics(rep):
 
 
 def main():
-    cfg, tag, reps = sys.argv[1], sys.argv[2], sys.argv[3:]
+    dry = "--dry" in sys.argv
+    args = [a for a in sys.argv[1:] if a != "--dry"]
+    cfg, tag, reps = args[0], args[1], args[2:]
     head = subprocess.run(["git", "rev-parse", "--short=12", "HEAD"], capture_output=True, text=True, cwd=ROOT).stdout.strip()
     path = os.path.join(ROOT, "profiles", "traffic.json")
     db = {}
@@ -68,7 +70,9 @@ def main():
                 continue
             ent[k] = {"bytes": int(b), "ncu_ms": round(ms, 4), "kernel": name[:120],
                       "source": f"{tag}: {os.path.basename(rep)} (ncu --set full, built from {head})"}
-            print(f"{cfg} {k:14s} {b / 1e9:9.3f} GB  {ms:9.3f} ms  {name[:80]}")
+            print(f"{cfg} {k:14s} {b / 1e9:9.3f} GB  {ms:9.3f} ms  {int(b)} {name[:80]}")
+    if dry:   # print only (GPU side); profiles/traffic.json is written from the printed lines
+        return
     with open(path, "w") as f:
         json.dump(db, f, indent=1, sort_keys=True)
 
