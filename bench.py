@@ -285,7 +285,44 @@ def run_speck(args):
 
     cfg = args.config
     t_gen = time.time()
-    probs = make_problems(cfg, dev)
+    t_bcast_ms = None
+    if world == 1:
+        probs = make_problems(cfg, dev)
+    else:
+        # rank 0 builds the inputs; every other rank receives them with the partitioner's
+        # broadcast_csr (the NCCL replication step of SURVEY §8(e)); timed with CUDA events
+        probs0 = make_problems(cfg, dev) if rank == 0 else None
+        torch.cuda.synchronize()
+        dist.barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        probs, seen = [], {}
+        n_probs = 2 if cfg == "c2" else 1
+        for j in range(n_probs):
+            label = probs0[j][0] if rank == 0 else ("A*P", "R*(AP)")[j] if cfg == "c2" else "A*A"
+            mats = []
+            for which in (1, 2):
+                M = probs0[j][which] if rank == 0 else None
+                key = id(M) if rank == 0 else (j, which)
+                has = torch.tensor([1 if (rank != 0 or M is not None) else 0], device=dev)
+                dist.broadcast(has, 0)
+                if not int(has.item()):
+                    mats.append(None)
+                    continue
+                same = torch.tensor([1 if (rank == 0 and which == 2 and M is probs0[j][1]) else 0], device=dev)
+                dist.broadcast(same, 0)
+                if int(same.item()):
+                    mats.append(mats[0])
+                    continue
+                R = sdist.broadcast_csr(M, src=0, device=dev)
+                mats.append(W.CSR(R.rows, R.cols, R.row_ptr, R.col, R.val))
+            probs.append((label, mats[0], mats[1]))
+        e1.record()
+        torch.cuda.synchronize()
+        t = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        t_bcast_ms = float(t.item())
+        del probs0
     torch.cuda.synchronize()
     log(f"[bench] generated {cfg} in {time.time() - t_gen:.1f}s")
     dtype = probs[0][1].dtype
@@ -479,7 +516,8 @@ def run_speck(args):
         for h in handles:
             h.close()
         torch.cuda.empty_cache()
-        e2e = run_e2e(sp, probs, dev, min(args.steps, 5), step_products, compute, world)
+        e2e = run_e2e(sp, probs, dev, min(args.steps, 5), step_products, compute, world,
+                      chunk_frac=args.e2e_chunk if cfg in ("c3", "c5") else 0.0)
 
     if rank == 0:
         out = {
@@ -494,6 +532,8 @@ def run_speck(args):
                        "model_GBps": round(model_step / (ms_per_step * 1e-3) / 1e9, 1),
                        "parallelism": f"row-sharded x{world}" if world > 1 else "single GPU",
                        "peak_mem_gb": round(peak_mem / 1e9, 3),
+                       "t_bcast_ms": None if t_bcast_ms is None else round(t_bcast_ms, 3),
+                       "ms_per_step_with_bcast": None if t_bcast_ms is None else round(ms_per_step + t_bcast_ms, 4),
                        "workspace_gb": round(sum(s["workspace_bytes"] for s in stats) / 1e9, 3),
                        "stage_ms": {probs[j][0]: {k[3:]: round(statistics.mean(v_), 4) for (jj, k), v_ in stage_ms.items()
                                                   if jj == j} for j in range(len(probs))},
@@ -512,51 +552,111 @@ def run_speck(args):
 E2E_STAGING_BYTES = 2 << 30
 
 
-def run_e2e(sp, probs, dev, steps, step_products, compute, world):
+def run_e2e(sp, probs, dev, steps, step_products, compute, world, chunk_frac=0.0):
     """Same metric through the public API, host (pinned) inputs in, host result out.  At N>1
     every rank copies the replicated inputs and reads back its own row block of the result;
-    the time is the max over ranks."""
+    the time is the max over ranks.
+
+    chunk_frac > 0 (single GPU, one product): the memory-bounded API (speck_row_chunks +
+    speck_spgemm_rows) with chunks of about chunk_frac of nnz(C) in two device
+    buffers; the D2H copy of chunk i (copy stream) overlaps the numeric work of chunk i+1, so
+    device C never exceeds 2 * chunk_frac of the full result."""
     host_in = []
     for (label, A, B) in probs:
-        host_in.append(tuple(None if M is None else W.CSR(M.rows, M.cols, M.row_ptr.cpu().pin_memory(),
-                                                           M.col.cpu().pin_memory(), M.val.cpu().pin_memory())
-                             for M in (A, B)))
-    dev_in = [tuple(None if M is None else W.CSR(M.rows, M.cols, torch.empty_like(M.row_ptr, device=dev),
-                                                 torch.empty_like(M.col, device=dev), torch.empty_like(M.val, device=dev))
-                    for M in pair) for pair in host_in]
+        hA = None if A is None else W.CSR(A.rows, A.cols, A.row_ptr.cpu().pin_memory(), A.col.cpu().pin_memory(),
+                                          A.val.cpu().pin_memory())
+        # A*A: B is the same matrix — one copy of the input crosses the link
+        hB = None if B is None else (hA if B is A else W.CSR(B.rows, B.cols, B.row_ptr.cpu().pin_memory(),
+                                                              B.col.cpu().pin_memory(), B.val.cpu().pin_memory()))
+        host_in.append((hA, hB))
+    dev_in = []
+    for hA, hB in host_in:
+        dA = None if hA is None else W.CSR(hA.rows, hA.cols, torch.empty_like(hA.row_ptr, device=dev),
+                                           torch.empty_like(hA.col, device=dev), torch.empty_like(hA.val, device=dev))
+        dB = None if hB is None else (dA if hB is hA else W.CSR(hB.rows, hB.cols, torch.empty_like(hB.row_ptr, device=dev),
+                                                                torch.empty_like(hB.col, device=dev),
+                                                                torch.empty_like(hB.val, device=dev)))
+        dev_in.append((dA, dB))
+    uniq = []
+    for (hA, hB), (dA, dB) in zip(host_in, dev_in):
+        for Mh, Md in ((hA, dA), (hB, dB)):
+            if Mh is not None and all(Mh is not u[0] for u in uniq):
+                uniq.append((Mh, Md))
     h = [sp.Handle(dev.index) for _ in probs]
-    bi = sum(t.numel() * t.element_size() for pair in host_in for M in pair if M is not None
-             for t in (M.row_ptr, M.col, M.val))
+    bi = sum(t.numel() * t.element_size() for Mh, _ in uniq for t in (Mh.row_ptr, Mh.col, Mh.val))
     stream = torch.cuda.current_stream()
-    times, bo, res = [], 0, None
+    copy_stream = torch.cuda.Stream(device=dev)
+    chunked = chunk_frac > 0 and world == 1 and len(probs) == 1
+    times, bo, res, chunk_info = [], 0, None, None
     for it in range(steps + 1):
         torch.cuda.synchronize()
         if world > 1:
             dist.barrier()
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         a.record(stream)
-        for pair_h, pair_d in zip(host_in, dev_in):
-            for Mh, Md in zip(pair_h, pair_d):
-                if Mh is None:
+        for Mh, Md in uniq:
+            Md.row_ptr.copy_(Mh.row_ptr, non_blocking=True)
+            Md.col.copy_(Mh.col, non_blocking=True)
+            Md.val.copy_(Mh.val, non_blocking=True)
+        if res is None:                                # pinned staging buffer (C3/C5 results are 70-90 GB,
+            res = torch.empty(E2E_STAGING_BYTES, dtype=torch.uint8, pin_memory=True)   # more than the host can pin)
+        if chunked:
+            (A, B), = dev_in
+            hd = h[0]
+            rp, nnz = hd.analyze(A, B)
+            maxrow = int(hd.stats()["max_row_products"])
+            budget = max(int(nnz * chunk_frac) + 1, maxrow + 1)
+            bounds = hd.row_chunks(rp, budget)
+            offs = rp[torch.tensor(bounds, device=dev)].cpu().tolist()     # one D2H for every chunk's range
+            cap = max(b_ - a_ for a_, b_ in zip(offs[:-1], offs[1:]))
+            bufs = [(torch.empty(cap, dtype=torch.int32, device=dev), torch.empty(cap, dtype=A.val.dtype, device=dev))
+                    for _ in range(2)]
+            done = [torch.cuda.Event(), torch.cuda.Event()]
+            copied = [None, None]
+            bo = rp.numel() * 8
+            pos = 0
+            # row_ptr first (the caller's copy of the structure), then the chunks
+            outs_rp = rp.view(torch.uint8)
+            with torch.cuda.stream(copy_stream):
+                copy_stream.wait_stream(stream)
+                for o in range(0, outs_rp.numel(), res.numel()):
+                    n = min(res.numel(), outs_rp.numel() - o)
+                    res[:n].copy_(outs_rp[o:o + n], non_blocking=True)
+            k = 0
+            for (r0, r1), (o0, o1) in zip(zip(bounds[:-1], bounds[1:]), zip(offs[:-1], offs[1:])):
+                if r1 <= r0:
                     continue
-                Md.row_ptr.copy_(Mh.row_ptr, non_blocking=True)
-                Md.col.copy_(Mh.col, non_blocking=True)
-                Md.val.copy_(Mh.val, non_blocking=True)
-        C = compute(dev_in, h)[-1]
-        outs = [t.view(torch.uint8) for t in (C.row_ptr, C.col, C.val) if t.numel()]
-        if res is None:                                # first (untimed) iteration: pinned staging buffer
-            # the result is streamed through a bounded pinned buffer (C3/C5 results are 70-90 GB,
-            # more than the host can pin); every byte of C still crosses PCIe/C2C each step
-            res = torch.empty(min(sum(t.numel() for t in outs), E2E_STAGING_BYTES), dtype=torch.uint8,
-                              pin_memory=True)
-        for t in outs:
-            for o in range(0, t.numel(), res.numel()):
-                n = min(res.numel(), t.numel() - o)
-                res[:n].copy_(t[o:o + n], non_blocking=True)
+                n_e = o1 - o0
+                col, val = bufs[k % 2]
+                if copied[k % 2] is not None:
+                    stream.wait_event(copied[k % 2])   # the buffer's previous chunk has left the device
+                hd.numeric_rows(A, B, rp, r0, r1, col[:n_e], val[:n_e])
+                done[k % 2].record(stream)
+                with torch.cuda.stream(copy_stream):
+                    copy_stream.wait_event(done[k % 2])
+                    for t in (col[:n_e].view(torch.uint8), val[:n_e].view(torch.uint8)):
+                        for o in range(0, t.numel(), res.numel()):
+                            n = min(res.numel(), t.numel() - o)
+                            res[:n].copy_(t[o:o + n], non_blocking=True)
+                    ev = torch.cuda.Event()
+                    ev.record(copy_stream)
+                    copied[k % 2] = ev
+                bo += n_e * (4 + A.val.element_size())
+                k += 1
+            stream.wait_stream(copy_stream)
+            chunk_info = {"chunks": k, "budget_entries": budget, "device_C_fraction": round(2 * cap / max(nnz, 1), 4)}
+            del bufs
+        else:
+            C = compute([(dA, dB) for dA, dB in dev_in], h)[-1]
+            outs = [t.view(torch.uint8) for t in (C.row_ptr, C.col, C.val) if t.numel()]
+            for t in outs:
+                for o in range(0, t.numel(), res.numel()):
+                    n = min(res.numel(), t.numel() - o)
+                    res[:n].copy_(t[o:o + n], non_blocking=True)
+            bo = sum(t.numel() for t in outs)
+            del C, outs                                # the next step's C must not coexist with this one
         b.record(stream)
         torch.cuda.synchronize()
-        bo = sum(t.numel() for t in outs)
-        del C, outs                                    # the next step's C must not coexist with this one
         if it > 0:                                     # first iteration warms the handles
             times.append(a.elapsed_time(b))
     ms = statistics.mean(times)
@@ -564,8 +664,11 @@ def run_e2e(sp, probs, dev, steps, step_products, compute, world):
         t = torch.tensor([ms], dtype=torch.float64, device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         ms = float(t.item())
-    return {"value": round(2.0 * step_products / (ms * 1e-3) / 1e9, 3), "unit": "GFLOP/s",
-            "h2d_bytes_per_step": int(bi), "d2h_bytes_per_step": int(bo), "ms_per_step": round(ms, 3)}
+    out = {"value": round(2.0 * step_products / (ms * 1e-3) / 1e9, 3), "unit": "GFLOP/s",
+           "h2d_bytes_per_step": int(bi), "d2h_bytes_per_step": int(bo), "ms_per_step": round(ms, 3)}
+    if chunked:
+        out["memory_bounded"] = chunk_info
+    return out
 
 
 # --------------------------------------------------------------------------- reference arm
@@ -611,6 +714,8 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--opt", action="append", default=[], help="library option name=value (experiments)")
     ap.add_argument("--cpu-budget", type=float, default=20.0, help="seconds of oracle work for the CPU baseline")
+    ap.add_argument("--e2e-chunk", type=float, default=0.125,
+                    help="c3/c5 e2e: memory-bounded chunks of this fraction of nnz(C) (0: one-shot)")
     args = ap.parse_args()
     if args.warmup < 3:
         log("[bench] warmup raised to 3 (timing rules)")

@@ -84,7 +84,10 @@ typedef enum {
   SPECK_OPT_STAGE_TIMING = 4,       /* 1: record per-stage times with CUDA events (syncs) [0] */
   SPECK_OPT_VALIDATE = 5,           /* 1: validate input CSR (sorted, unique, in range) [0] */
   SPECK_OPT_DISABLE_DIRECT = 6,     /* 1: route single-NZ rows through the accumulators [0] */
-  SPECK_OPT_FIXED_GROUP_SIZE = 7,   /* >0: use this g for every block instead of the local LB [0] */
+  SPECK_OPT_FIXED_GROUP_SIZE = 7,   /* local load balancing of hash rows: 0 expand-balanced (every lane
+                                       the same number of products, B200 default); >0 the paper's groups of g
+                                       threads per referenced B row with this fixed g (power of two, clamped to the
+                                       row's threads); -1 the paper's dynamic g (reading R9) [0] */
   SPECK_OPT_CONCURRENT_STREAMS = 8, /* number of internal streams for concurrent bins, 1..8 [4] */
   SPECK_OPT_SEGMENTS = 9,           /* 1: split rows beyond the largest map into column segments; 0: windowed dense [1] */
   SPECK_OPT_WARP_ROWS = 10,         /* 1: smallest bin = one warp per row (k_warp_rows); 0: merged blocks (Alg. 2) [1] */
@@ -95,9 +98,13 @@ typedef enum {
                                        by speck_get_stats (kernel_id / kernel_bin / kernel_ms) [0] */
   SPECK_OPT_PATH_COUNTERS = 14,     /* 1: count the rows each accumulator path processes (path_rows); costs a few
                                        atomics per row — tests and diagnostics only [0] */
-  SPECK_OPT_BUCKET_SORT = 15        /* rows whose products are mostly distinct columns use a counting sort on
+  SPECK_OPT_BUCKET_SORT = 15,       /* rows whose products are mostly distinct columns use a counting sort on
                                        column buckets instead of the hash map: 0 off, 1 numeric rows, 2 numeric
                                        and symbolic rows [1] */
+  SPECK_OPT_DETERMINISTIC = 16      /* 1: every row of C accumulated by one warp in the order of eq. (1)'s sum, each
+                                       product rounded before it is added: values bit-identical across runs and
+                                       equal to a sequential sum in the inputs' precision (reading R15); slower
+                                       for large rows [0] */
 } speck_option_t;
 /* Changing any option except STAGE_TIMING, CONCURRENT_STREAMS, GLOBAL_LB_NUMERIC, VALIDATE,
  * KERNEL_TIMING and PATH_COUNTERS after speck_analyze invalidates the analysis: the next
@@ -144,6 +151,7 @@ typedef enum {
   SPECK_PATH_NUM_ESC = 20,        /* numeric bucket counting sort, no repeated column */
   SPECK_PATH_NUM_ESC_DUP = 21,    /* numeric bucket counting sort with repeated columns */
   SPECK_PATH_ESC_FALLBACK = 22,   /* bucket counting sort abandoned (uneven buckets): hash map instead */
+  SPECK_PATH_NUM_DET = 23,        /* deterministic mode: one warp per large row (k_det_rows) */
   SPECK_PATH_COUNT = 24
 } speck_path_t;
 
@@ -274,9 +282,11 @@ const char* speck_last_error(speck_handle_t handle);
 const char* speck_version(void);
 
 /* ----------------------------------------------------------------------------------
- * Component entry points.  They run the SAME device functions the pipeline uses, on
- * device buffers, so the paper's worked examples and the plan logic can be checked
- * against the oracle in isolation.  All asynchronous on `stream`.
+ * Component entry points: each runs, on device buffers, a device function the pipeline
+ * itself calls (warp_block_merge in the merged-block kernels, local_group_size in the
+ * SPECK_OPT_FIXED_GROUP_SIZE = -1 expansion, probe_insert_mono in the numeric maps of
+ * scrambled rows, the look-back scan of the C row offsets), so the paper's worked examples can
+ * be checked against the oracle in isolation.  All asynchronous on `stream`.
  * ---------------------------------------------------------------------------------- */
 
 /* Block merge (Alg. 2; Fig. 3), reading R10: for each aligned group

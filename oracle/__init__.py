@@ -43,6 +43,7 @@ def lib():
         L.oracle_row_analysis.argtypes = [I64, P, P, P, P, P, P, P, P, P]
         L.oracle_symbolic.argtypes = [P, P, P, P, I64, I64, I64, P]
         L.oracle_numeric.argtypes = [P, P, P, P, P, P, ctypes.c_int, I64, I64, I64, P, P, P, P]
+        L.oracle_numeric_sequential.argtypes = [P, P, P, P, P, P, ctypes.c_int, I64, I64, I64, P, P, P]
         L.oracle_block_merge.argtypes = [I64, P, I64, ctypes.c_int, P, P]
         L.oracle_block_merge.restype = I64
         L.oracle_group_iters.argtypes = [I64, P, I64, I64]
@@ -132,6 +133,26 @@ def spgemm(A, B, r0: int = 0, r1: Optional[int] = None, with_scale: bool = True)
     if err:
         raise RuntimeError(f"oracle_numeric error {err}")
     return rp, col, val, scale
+
+
+def spgemm_sequential(A, B, r0: int = 0, r1: Optional[int] = None):
+    """C = A·B rows [r0, r1) with every sum taken left to right in the inputs' precision, each
+    product rounded before it is added (reading R15; the deterministic mode's exact bits).
+    Returns (row_ptr, col, val as float64 holding the fp32/fp64 results)."""
+    m, k, arp, acol, aval = _host(A)
+    kb, n, brp, bcol, bval = _host(B)
+    assert k == kb and aval.dtype == bval.dtype
+    is64 = 1 if aval.dtype == np.float64 else 0
+    r1 = m if r1 is None else r1
+    cnt = symbolic((m, k, arp, acol, aval), (kb, n, brp, bcol, bval), r0, r1)
+    rp = np.zeros(r1 - r0 + 1, np.int64)
+    np.cumsum(cnt, out=rp[1:])
+    col = np.empty(int(rp[-1]), np.int32); val = np.empty(int(rp[-1]), np.float64)
+    err = lib().oracle_numeric_sequential(_p(arp), _p(acol), _p(aval), _p(brp), _p(bcol), _p(bval), is64, n, r0, r1,
+                                          _p(rp), _p(col), _p(val))
+    if err:
+        raise RuntimeError(f"oracle_numeric_sequential error {err}")
+    return rp, col, val
 
 
 def block_merge(needs, cap: int, levels: int = 5):

@@ -15,6 +15,8 @@
  *   oracle_symbolic       structural nnz per C row (eq. (1))
  *   oracle_numeric        C = A·B, eq. (1), rows sorted by column (P:98-103,
  *                         P:1121-1123); structural zeros kept (R1)
+ *   oracle_numeric_sequential  the same sums left to right in the inputs' precision
+ *                         (deterministic-value mode, R15)
  *   oracle_block_merge    Algorithm 2 + Fig. 3, reading R10
  *   oracle_group_iters    Fig. 1 iteration model
  *   oracle_group_size     local load balancer g, reading R9
@@ -227,6 +229,67 @@ int oracle_numeric(const int64_t *A_rp, const int32_t *A_col, const void *A_val,
             }
         }
         scratch_free(&s);
+    }
+    return err;
+}
+
+/* Sequential working-precision values (deterministic-value mode; DESIGN.md
+ * reading R15): C_ij accumulated left to right in the order of eq. (1)'s sum — k in the order
+ * of row i of A, then the entries of B_k in order — in the inputs' own precision, every
+ * product rounded before it is added:  acc <- fl(acc + fl(A_ik * B_kj)), acc starting at the
+ * first product.  (The library's deterministic mode promises exactly these bits.)  Structure as
+ * oracle_numeric; out_val is the float / double result widened to double. */
+int oracle_numeric_sequential(const int64_t *A_rp, const int32_t *A_col, const void *A_val,
+                              const int64_t *B_rp, const int32_t *B_col, const void *B_val, int is_f64,
+                              int64_t ncols, int64_t r0, int64_t r1, const int64_t *out_rp,
+                              int32_t *out_col, double *out_val) {
+    int err = ORACLE_OK;
+#pragma omp parallel
+    {
+        int64_t *mark = (int64_t *)malloc(sizeof(int64_t) * (size_t)(ncols > 0 ? ncols : 1));
+        double *accd = (double *)malloc(sizeof(double) * (size_t)(ncols > 0 ? ncols : 1));
+        float *accf = (float *)malloc(sizeof(float) * (size_t)(ncols > 0 ? ncols : 1));
+        int32_t *touched = (int32_t *)malloc(sizeof(int32_t) * (size_t)(ncols > 0 ? ncols : 1));
+        int my = (mark && accd && accf && touched) ? ORACLE_OK : ORACLE_ERR_ALLOC;
+        if (my != ORACLE_OK) {
+#pragma omp atomic write
+            err = my;
+        } else {
+            for (int64_t j = 0; j < ncols; ++j) mark[j] = -1;
+        }
+#pragma omp for schedule(dynamic, 1024)
+        for (int64_t i = r0; i < r1; ++i) {
+            if (my != ORACLE_OK) continue;
+            int64_t n = 0;
+            for (int64_t p = A_rp[i]; p < A_rp[i + 1]; ++p) {
+                int32_t k = A_col[p];
+                for (int64_t q = B_rp[k]; q < B_rp[k + 1]; ++q) {
+                    int32_t j = B_col[q];
+                    if (is_f64) {
+                        volatile double prod = ((const double *)A_val)[p] * ((const double *)B_val)[q];
+                        if (mark[j] != i) { mark[j] = i; accd[j] = prod; touched[n++] = j; }
+                        else accd[j] = accd[j] + prod;
+                    } else {
+                        volatile float prod = ((const float *)A_val)[p] * ((const float *)B_val)[q];
+                        if (mark[j] != i) { mark[j] = i; accf[j] = prod; touched[n++] = j; }
+                        else accf[j] = accf[j] + prod;
+                    }
+                }
+            }
+            qsort(touched, (size_t)n, sizeof(int32_t), cmp_i32);
+            int64_t base = out_rp[i - r0];
+            if (out_rp[i - r0 + 1] - base != n) {
+#pragma omp atomic write
+                err = ORACLE_ERR_ARG;
+                continue;
+            }
+            for (int64_t t = 0; t < n; ++t) {
+                int32_t j = touched[t];
+                out_col[base + t] = j;
+                out_val[base + t] = is_f64 ? accd[j] : (double)accf[j];
+            }
+        }
+        free(mark); free(accd); free(accf); free(touched);
     }
     return err;
 }

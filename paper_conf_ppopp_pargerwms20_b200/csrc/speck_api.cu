@@ -17,6 +17,7 @@
 #include "spgemm_kernels.cuh"
 #include "segment_kernels.cuh"
 #include "transpose_kernels.cuh"
+#include "det_kernels.cuh"
 
 #define SPECK_VERSION "speck-b200 0.1.0 (sm_100a)"
 
@@ -53,7 +54,7 @@ struct speck_handle_s {
   std::string err;
   // options
   int64_t opt_lb_sym = -1, opt_lb_num = -1, opt_force_acc = 0, opt_dense_window = 0, opt_timing = 0, opt_validate = 0,
-          opt_disable_direct = 0, opt_fixed_g = 0, opt_streams = 4, opt_esc = 1;
+          opt_disable_direct = 0, opt_fixed_g = 0, opt_streams = 4, opt_esc = 1, opt_det = 0;
   // workspace
   Buf prods, maxlen, colmin, colmax, cnt, hist, hist_off, bins, stats, scan_status, resume, small, ana_long, binfo;
   unsigned long long* h_pinned = nullptr;  // pinned readback area (kPinnedWords x u64)
@@ -83,7 +84,7 @@ struct speck_handle_s {
   bool seg_enabled = false;
   int seg_shift = 15, nchunks = 0;
   int64_t long_thr = INT64_MAX, n_cand = 0, n_segs = 0, cand_start = 0;
-  Buf chunk_cnt, cand, nseg, seg_off, segs, chunks, tr_cnt, tr_list, tr_col, tr_val;
+  Buf chunk_cnt, cand, nseg, seg_off, segs, chunks, tr_cnt, tr_list, tr_col, tr_val, det_scratch;
   // SPECK_OPT_KERNEL_TIMING: one event pair per launch of the current analyze/spgemm pair
   int64_t opt_ktime = 0, opt_paths = 0;
   cudaEvent_t kt_ev[2 * kMaxTimed] = {};
@@ -177,7 +178,7 @@ int64_t ws_bytes(speck_handle_t h) {
                    h->hist_off.cap + h->bins.cap + h->stats.cap + h->scan_status.cap + h->resume.cap + h->small.cap +
                    h->ana_long.cap + h->chunk_cnt.cap + h->cand.cap + h->nseg.cap + h->seg_off.cap + h->segs.cap +
                    h->bm_pool.cap + h->bm_off.cap + h->binfo.cap + h->paths.cap + h->chunks.cap +
-                   h->tr_cnt.cap + h->tr_list.cap + h->tr_col.cap + h->tr_val.cap);
+                   h->tr_cnt.cap + h->tr_list.cap + h->tr_col.cap + h->tr_val.cap + h->det_scratch.cap);
 }
 
 speck_status_t check_csr(speck_handle_t h, const speck_csr_t* M, const char* name, bool need_values) {
@@ -278,6 +279,7 @@ speck_status_t set_smem_attrs(speck_handle_t h) {
       CK(cudaFuncSetAttribute(spgemm_fn<V>(c, pass), cudaFuncAttributeMaxDynamicSharedMemorySize, kCfgMapBytes[c]));
   CK(cudaFuncSetAttribute(k_segments<V>, cudaFuncAttributeMaxDynamicSharedMemorySize, kCfgMapBytes[kSegCfg]));
   CK(cudaFuncSetAttribute(k_tr_sort_block<V>, cudaFuncAttributeMaxDynamicSharedMemorySize, kTrSmemSort * (4 + (int)sizeof(V))));
+  CK(cudaFuncSetAttribute(k_det_rows<V>, cudaFuncAttributeMaxDynamicSharedMemorySize, kDetRegion * kDetWarps));
   CK(cudaFuncSetAttribute(k_long_bitmap<V>, cudaFuncAttributeMaxDynamicSharedMemorySize, kCfgMapBytes[kNumCfg - 1]));
   CK(cudaFuncSetAttribute(k_warp_rows<0, V, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytesSym * (kWarpRowThreads / 32)));
   CK(cudaFuncSetAttribute(k_warp_rows<0, V, 3>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytesSym * (kWarpRowThreads / 32)));
@@ -374,7 +376,7 @@ void plan_segments(speck_handle_t h, int64_t ncols) {
   while ((int64_t)1 << (s + 1) <= num_dense_window<V>(kSegCfg)) ++s;
   h->seg_shift = s;
   h->nchunks = (int)((ncols + ((int64_t)1 << s) - 1) >> s);
-  h->seg_enabled = h->opt_force_acc != 2 && h->opt_segments != 0 && h->nchunks >= 1 && h->nchunks <= kMaxChunks;
+  h->seg_enabled = h->opt_force_acc != 2 && h->opt_segments != 0 && !h->opt_det && h->nchunks >= 1 && h->nchunks <= kMaxChunks;
   h->n_cand = 0;
   h->n_segs = 0;
 }
@@ -409,7 +411,8 @@ SpgemmArgs<V> base_args(speck_handle_t h, const speck_csr_t* A, const speck_csr_
   a.force_acc = (int)h->opt_force_acc;
   a.dense_window_cap = h->opt_dense_window;
   a.fixed_g = (int)h->opt_fixed_g;
-  a.esc = (int)h->opt_esc;
+  a.esc = h->opt_det ? 0 : (int)h->opt_esc;          // deterministic: one warp per row, in-order adds
+  if (h->opt_det) a.fixed_g = 0;
   a.paths = h->opt_paths ? static_cast<unsigned long long*>(h->paths.p) : nullptr;
   a.row_lo = 0;
   a.row_hi = INT64_MAX;
@@ -537,6 +540,20 @@ speck_status_t run_pass(speck_handle_t h, int pass, int lb, const int64_t* cat_b
     SpgemmArgs<V> b = a;
     b.rows = bins + cat_beg[cat];
     b.n_entries = n;
+    if (pass == 1 && h->opt_det && (c > 0 || !h->opt_warp_rows)) {
+      // deterministic mode: rows beyond the warp region -> one warp per row (det_kernels.cuh)
+      const int64_t slots = (int64_t)h->num_sms * kDetWarps;
+      if ((st = ensure(h, h->det_scratch, (size_t)slots * (size_t)a.resume_stride * 4, h->streams[si]))) return st;
+      unsigned long long* ctr = reinterpret_cast<unsigned long long*>(static_cast<char*>(h->small.p) + 1280 + 8 * c);
+      CK(cudaMemsetAsync(ctr, 0, 8, h->streams[si]));
+      const int kt = kt_begin(h, h->streams[si], SPECK_KERNEL_NUM_BLOCK, c, 16 + cat);
+      k_det_rows<V><<<(unsigned)std::min<int64_t>(h->num_sms, (n + kDetWarps - 1) / kDetWarps), 32 * kDetWarps,
+                      (size_t)kDetRegion * kDetWarps, h->streams[si]>>>(b, ctr, static_cast<int32_t*>(h->det_scratch.p));
+      CKL();
+      kt_end(h, h->streams[si], kt);
+      si = (si + 1) % ns;
+      continue;
+    }
     if (c == 0 && h->opt_warp_rows) {
       st = launch_warp_rows<V>(h, pass, b, h->streams[si], pass == 1 ? 2 : 0, pass * 16 + cat);
       if (st) return st;
@@ -974,7 +991,7 @@ speck_status_t spgemm_impl(speck_handle_t h, const speck_csr_t* A, const speck_c
   const BinParams bpn = make_bin_params(h, 1);
   const int cfg_max = cfg_for(bpn, h->max_cnt);
   const int lb = decide_lb(kLbNum, h->opt_lb_num, (double)h->max_cnt, (double)h->nnz_c, m, cfg_max,
-                           cfg_max >= kNumCfg - 1 || h->opt_force_acc == 2);
+                           cfg_max >= kNumCfg - 1 || h->opt_force_acc == 2 || h->opt_det);
   h->st.lb_numeric = lb;
   h->lb_num = lb;
   if ((st = timing_mark(h, 5, s))) return st;
@@ -1126,7 +1143,7 @@ speck_status_t speck_destroy(speck_handle_t h) {
   Buf* bufs[] = {&h->prods, &h->maxlen, &h->colmin, &h->colmax, &h->cnt, &h->hist, &h->hist_off, &h->bins, &h->stats,
                  &h->scan_status, &h->resume, &h->small, &h->ana_long, &h->chunk_cnt, &h->cand, &h->nseg,
                  &h->seg_off, &h->segs, &h->bm_pool, &h->bm_off, &h->binfo, &h->paths, &h->chunks, &h->tr_cnt,
-                 &h->tr_list, &h->tr_col, &h->tr_val};
+                 &h->tr_list, &h->tr_col, &h->tr_val, &h->det_scratch};
   for (Buf* b : bufs) {
     if (!b->p) continue;
     if (h->urelease) h->urelease(b->p, nullptr, h->uctx);
@@ -1170,7 +1187,8 @@ speck_status_t speck_set_option(speck_handle_t h, int option, int64_t v) {
     case SPECK_OPT_VALIDATE: h->opt_validate = v; break;
     case SPECK_OPT_DISABLE_DIRECT: h->opt_disable_direct = v; break;
     case SPECK_OPT_FIXED_GROUP_SIZE:
-      if (v < 0 || v > 1024 || (v & (v - 1))) return fail(h, SPECK_ERR_INVALID_ARGUMENT, "FIXED_GROUP_SIZE must be 0 or a power of two <= 1024");
+      if (v < -1 || v > 1024 || (v > 0 && (v & (v - 1))))
+        return fail(h, SPECK_ERR_INVALID_ARGUMENT, "FIXED_GROUP_SIZE must be -1, 0 or a power of two <= 1024");
       h->opt_fixed_g = v; break;
     case SPECK_OPT_CONCURRENT_STREAMS:
       if (v < 1 || v > kMaxStreams) return fail(h, SPECK_ERR_INVALID_ARGUMENT, "CONCURRENT_STREAMS must be 1..8");
@@ -1180,6 +1198,7 @@ speck_status_t speck_set_option(speck_handle_t h, int option, int64_t v) {
     case SPECK_OPT_LONG_BITMAP: h->opt_long_bitmap = v; break;
     case SPECK_OPT_BITMAP_REUSE: h->opt_bitmap_reuse = v; break;
     case SPECK_OPT_KERNEL_TIMING: h->opt_ktime = v; break;
+    case SPECK_OPT_DETERMINISTIC: h->opt_det = v ? 1 : 0; break;
     case SPECK_OPT_BUCKET_SORT:
       if (v < 0 || v > 2) return fail(h, SPECK_ERR_INVALID_ARGUMENT, "BUCKET_SORT must be 0..2");
       h->opt_esc = v; break;
@@ -1345,7 +1364,7 @@ speck_status_t speck_set_allocator(speck_handle_t h, speck_alloc_fn alloc, speck
   Buf* bufs[] = {&h->prods, &h->maxlen, &h->colmin, &h->colmax, &h->cnt, &h->hist, &h->hist_off, &h->bins, &h->stats,
                  &h->scan_status, &h->resume, &h->small, &h->ana_long, &h->chunk_cnt, &h->cand, &h->nseg,
                  &h->seg_off, &h->segs, &h->bm_pool, &h->bm_off, &h->binfo, &h->paths, &h->chunks, &h->tr_cnt,
-                 &h->tr_list, &h->tr_col, &h->tr_val};
+                 &h->tr_list, &h->tr_col, &h->tr_val, &h->det_scratch};
   for (Buf* b : bufs) release_buf(h, *b, nullptr);
   cudaStreamSynchronize(nullptr);
   h->ualloc = alloc;

@@ -65,6 +65,10 @@ static_assert(cfg_fits<0>() && cfg_fits<1>() && cfg_fits<2>() && cfg_fits<3>() &
 
 template <typename V>
 __device__ __forceinline__ V ldv(const V* p) { return __ldg(p); }
+// a + b rounded once, never contracted with the product that produced b (in-order, per-product
+// rounded sums: the warp-per-row paths match oracle_numeric_sequential bit for bit)
+__device__ __forceinline__ float add_rn(float a, float b) { return __fadd_rn(a, b); }
+__device__ __forceinline__ double add_rn(double a, double b) { return __dadd_rn(a, b); }
 
 // Order-preserving numeric maps: 8-slot buckets, the home bucket monotone in the column over
 // the row's [colmin, colmax] and covering the first 7/8 of the buckets (the rest absorbs
@@ -471,6 +475,48 @@ __device__ __forceinline__ void expand_row(const SpgemmArgs<V>& p, int64_t a0, i
   }
 }
 
+// The paper's local load balancer: groups of g threads (g a power of two, 1..32*nw)
+// are assigned round-robin to the referenced B rows of the row of A; the g threads of a group
+// stride over their B row.  g = SPECK_OPT_FIXED_GROUP_SIZE, or the dynamic group
+// size of P:940-970 (local_group_size, reading R9) when the option is -1.  Kept for the Fig. 13
+// ablation and as an option; the default is the expand-balanced enumeration (expand_esc /
+// expand_row), which gives every lane the same number of products.  f(col, a*b, active) is
+// called by all 32 lanes of the warp in step.
+template <int PASS, typename V, typename F>
+__device__ __forceinline__ void expand_grouped(const SpgemmArgs<V>& p, int64_t a0, int alen, int wi, int nw, int g,
+                                               F&& f) {
+  const int lane = lane_id();
+  const int T = 32 * nw;
+  g = g < 1 ? 1 : (g > T ? T : g);
+  const int k = T / g;                                  // groups
+  const int tid = wi * 32 + lane;
+  const int q = tid / g, t = tid % g;                   // group, thread within the group
+  for (int r0 = 0; r0 < alen; r0 += k) {
+    const int fi = r0 + q;                              // this group's referenced row in the round
+    int64_t bst = 0;
+    int len = 0;
+    V a = V(0);
+    if (fi < alen) {
+      const int32_t kc = p.A_col[a0 + fi];
+      if (PASS == 1) a = __ldg(p.A_val + a0 + fi);
+      bst = p.B_rp[kc];
+      len = (int)(p.B_rp[kc + 1] - bst);
+    }
+    const int iters = (int)__reduce_max_sync(0xffffffffu, (unsigned)((len - t + g - 1) > 0 ? (len - t + g - 1) / g : 0));
+    for (int it = 0; it < iters; ++it) {
+      const int j = t + it * g;
+      const bool act = j < len;
+      uint32_t col = 0x80000000u | (uint32_t)lane;
+      V bv = V(0);
+      if (act) {
+        col = (uint32_t)p.B_col[bst + j];
+        if (PASS == 1) bv = __ldg(p.B_val + bst + j);
+      }
+      f(col, a * bv, act);
+    }
+  }
+}
+
 // Referenced B rows of at least kLongB entries collected into a shared list (collect_long_rows)
 // and streamed by all nw warps, product chunks rotated over the warps (no redundant batch
 // loads, unlike expand_row's ALL mode, which re-reads every batch in every warp: for C4's
@@ -746,7 +792,8 @@ __device__ __noinline__ void block_sorted_write(uint32_t* keys, V* vals, uint32_
 template <int PASS, typename V, int MODE = 0>
 __device__ __forceinline__ int warp_row(const SpgemmArgs<V>& p, uint32_t* rk, V* rv, uint32_t S, int64_t a0, int alen,
                                         int32_t cmin, int32_t cmax, int32_t cnt, int64_t cbase,
-                                        const PreBatch<V>* pre = nullptr) {
+                                        const PreBatch<V>* pre = nullptr, int64_t warp_row_prods = 0,
+                                        int64_t warp_row_maxlen = 0) {
   const int lane = lane_id();
   for (uint32_t i = lane; i < S; i += 32) {
     rk[i] = kEmptyKey;
@@ -779,13 +826,21 @@ __device__ __forceinline__ int warp_row(const SpgemmArgs<V>& p, uint32_t* rk, V*
       const int rank = __popc(peers & lt);
       const int maxg = (int)__reduce_max_sync(0xffffffffu, (unsigned)__popc(peers));
       for (int t = 0; t < maxg; ++t) {
-        if (act && rank == t) rv[s] += v;
+        if (act && rank == t) rv[s] = add_rn(rv[s], v);
         __syncwarp();
       }
     }
   };
-  if (PASS == 0) expand_row<PASS, V, true, false, 2>(p, a0, alen, 0, 1, ins);
-  else expand_esc<PASS, V, SPECK_WARP_U>(p, a0, alen, 0, 1, ins, pre);
+  if (p.fixed_g != 0) {
+    // the paper's local load balancing (Fig. 13 ablation): one warp = T threads, g per group
+    int g = p.fixed_g;
+    if (g < 0) g = local_group_size(32, alen, warp_row_prods, warp_row_maxlen);
+    expand_grouped<PASS, V>(p, a0, alen, 0, 1, g, ins);
+  } else if (PASS == 0) {
+    expand_row<PASS, V, true, false, 2>(p, a0, alen, 0, 1, ins);
+  } else {
+    expand_esc<PASS, V, SPECK_WARP_U>(p, a0, alen, 0, 1, ins, pre);
+  }
   if (PASS == 0) {
     if (lane == 0) count_path(p.paths, SPECK_PATH_SYM_WARP);
     return warp_sum(newc);
@@ -1002,8 +1057,7 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
         const uint64_t mmult = bkt_mult((uint32_t)(bm.rhi[r] - bm.rlo[r] + 1), S);
         const bool ordered = bm.ordered;
         int newc = 0, wrapped = 0;
-        expand_esc<PASS, V, PASS == 0 ? 4 : 2>(p, bm.astart[r], (int)(bm.aoff[r + 1] - bm.aoff[r]), warp_id(), NW,
-                            [&](uint32_t col, V v, bool act) {
+        auto ins = [&](uint32_t col, V v, bool act) {
                               if (PASS == 0) {
                                 if (act) newc += hash_insert_key(rk, S, col);
                               } else {
@@ -1015,7 +1069,16 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
                                 const V sum = warp_key_sum(col, v, leader);
                                 if (act && leader) atomicAdd(&rv[s], sum);
                               }
-                            });
+                            };
+        const int ralen = (int)(bm.aoff[r + 1] - bm.aoff[r]);
+        if (p.fixed_g != 0) {
+          // the paper's local load balancing (Fig. 13 ablation): T threads in groups of g
+          const int g = p.fixed_g > 0 ? p.fixed_g
+                                      : local_group_size(T, ralen, p.prods[bm.row[b0 + r]], p.maxlen[bm.row[b0 + r]]);
+          expand_grouped<PASS, V>(p, bm.astart[r], ralen, warp_id(), NW, g, ins);
+        } else {
+          expand_esc<PASS, V, PASS == 0 ? 4 : 2>(p, bm.astart[r], ralen, warp_id(), NW, ins);
+        }
         if (PASS == 0) {
           newc = warp_sum(newc);
           if (lane_id() == 0 && newc) atomicAdd(&bm.rcnt[r], newc);
@@ -1200,6 +1263,7 @@ __global__ void __launch_bounds__(kWarpRowThreads, wr_ctas_per_sm(PASS, MODE))
       else if (lane == 4 && kRange) mv = p.colmin[row];   // column range: ordered maps only
       else if (lane == 5 && kRange) mv = p.colmax[row];
       else if (lane == 6 && PASS == 1 && MODE != 1) mv = p.prods[row];
+      else if (lane == 7 && p.fixed_g < 0) mv = p.maxlen[row];     // dynamic g (paper's local LB)
     }
   };
   // rows are claimed kWarpRowChunk at a time (one same-address atomic per chunk: per-row
@@ -1281,7 +1345,10 @@ __global__ void __launch_bounds__(kWarpRowThreads, wr_ctas_per_sm(PASS, MODE))
       if (p.esc >= (PASS == 0 ? 2 : 1) && np > 0 && np <= esc_cap && (PASS == 0 || np <= 2 * need))
         c = esc_row<1, PASS, V>(p, region, kRegion, 0, a0, alen, (int)np, (int)need, cmn, cmx, m2, nullptr, nullptr, 0);
     }
-    if (c < 0) c = warp_row<PASS, V, MODE>(p, rk, rv, S, a0, alen, cmn, cmx, (int32_t)(m3 - m2), m2, &bcur);
+    if (c < 0)
+      c = warp_row<PASS, V, MODE>(p, rk, rv, S, a0, alen, cmn, cmx, (int32_t)(m3 - m2), m2, &bcur,
+                                  PASS == 0 ? need : __shfl_sync(0xffffffffu, mv_prev6, 6),
+                                  __shfl_sync(0xffffffffu, mv_prev6, 7));
     if (PASS == 0 && lane == 0) p.cnt[cur] = c;
     e = en;
     en = enn;

@@ -149,3 +149,78 @@ def allgather_csr(blk: RowBlock, m: int, group=None):
     col = torch.cat([c[:n] for c, (_, _, n) in zip(cols, metas)])
     val = torch.cat([v[:n] for v, (_, _, n) in zip(vals, metas)])
     return type("CSRG", (), dict(rows=m, cols=blk.cols, row_ptr=row_ptr, col=col, val=val))()
+
+
+# ------------------------------------------------------------------------------ 2-D grid
+# multi-GPU without full replication of B ("shared matrix storage in multi-GPU
+# setups").  Ranks form a pr x pc grid; rank (i, j) holds the row block A_i of A
+# and the column block B_:j of B (columns [c_j, c_{j+1}) renumbered from 0), so each GPU stores
+# 1/pc of B instead of all of it.  C_ij = A_i · B_:j is the (i, j) tile of C with local columns;
+# the row block C_i is the concatenation, row by row, of C_i0, C_i1, ... with columns shifted by
+# c_j (column blocks are disjoint and ordered, so the rows stay sorted).
+
+
+def column_block(B, c0: int, c1: int):
+    """Columns [c0, c1) of B renumbered from 0 (rows kept; the CSR slice rank (i, j) stores)."""
+    rows = torch.repeat_interleave(torch.arange(B.rows, device=B.col.device), B.row_ptr[1:] - B.row_ptr[:-1])
+    keep = (B.col >= c0) & (B.col < c1)
+    counts = torch.bincount(rows[keep], minlength=B.rows)
+    rp = torch.zeros(B.rows + 1, dtype=torch.int64, device=B.col.device)
+    rp[1:] = torch.cumsum(counts, 0)
+    return type("CSRCol", (), dict(rows=B.rows, cols=c1 - c0, row_ptr=rp, col=(B.col[keep] - c0).to(torch.int32),
+                                   val=B.val[keep]))()
+
+
+def column_bounds(ncols: int, parts: int) -> List[int]:
+    return [ncols * j // parts for j in range(parts + 1)]
+
+
+def grid_coords(rank: int, pc: int):
+    return divmod(rank, pc)
+
+
+def spgemm_2d_tile(A_i, B_j, local: Optional[Callable] = None):
+    """This rank's tile C_ij = A_i · B_:j (local columns)."""
+    return (local or _default_local)(A_i, B_j)
+
+
+def assemble_row_block(tile, c0: int, row_group, n_cols: int):
+    """Concatenate the tiles of one row block (all ranks of `row_group`, in column order) into
+    the rows of C_i with global columns; every rank of the row group receives C_i."""
+    world = dist.get_world_size(row_group)
+    dev = tile.row_ptr.device
+    m = tile.row_ptr.numel() - 1
+    meta = torch.tensor([c0, tile.col.numel()], dtype=torch.int64, device=dev)
+    metas = [torch.zeros_like(meta) for _ in range(world)]
+    dist.all_gather(metas, meta, group=row_group)
+    metas = [tuple(int(v) for v in x.tolist()) for x in metas]
+    lens = [torch.empty(m, dtype=torch.int64, device=dev) for _ in range(world)]
+    dist.all_gather(lens, (tile.row_ptr[1:] - tile.row_ptr[:-1]).contiguous(), group=row_group)
+    mx = max(n for _, n in metas)
+    cols, vals = [], []
+    for t, src in ((tile.col, cols), (tile.val, vals)):
+        buf = torch.zeros(max(mx, 1), dtype=t.dtype, device=dev)
+        buf[:t.numel()] = t
+        outs = [torch.empty(max(mx, 1), dtype=t.dtype, device=dev) for _ in range(world)]
+        dist.all_gather(outs, buf, group=row_group)
+        src.extend(outs)
+    order = sorted(range(world), key=lambda q: metas[q][0])       # column order
+    total = sum(lens)
+    rp = torch.zeros(m + 1, dtype=torch.int64, device=dev)
+    rp[1:] = torch.cumsum(total, 0)
+    nnz = int(rp[-1])
+    col = torch.empty(nnz, dtype=torch.int32, device=dev)
+    val = torch.empty(nnz, dtype=tile.val.dtype, device=dev)
+    before = torch.zeros(m, dtype=torch.int64, device=dev)        # entries of earlier column blocks per row
+    for q in order:
+        c0q, nq = metas[q]
+        lq = lens[q]
+        rows = torch.repeat_interleave(torch.arange(m, device=dev), lq)
+        start = torch.zeros(m + 1, dtype=torch.int64, device=dev)
+        start[1:] = torch.cumsum(lq, 0)
+        t_in_row = torch.arange(nq, device=dev) - start[rows]
+        dst = rp[rows] + before[rows] + t_in_row
+        col[dst] = cols[q][:nq] + c0q
+        val[dst] = vals[q][:nq]
+        before += lq
+    return type("CSRRow", (), dict(rows=m, cols=n_cols, row_ptr=rp, col=col, val=val))()

@@ -24,7 +24,7 @@ OPT = {
     "global_lb_symbolic": 0, "global_lb_numeric": 1, "force_accumulator": 2, "dense_window": 3,
     "stage_timing": 4, "validate": 5, "disable_direct": 6, "fixed_group_size": 7, "concurrent_streams": 8,
     "segments": 9, "warp_rows": 10, "long_bitmap": 11, "bitmap_reuse": 12, "kernel_timing": 13,
-    "path_counters": 14, "bucket_sort": 15,
+    "path_counters": 14, "bucket_sort": 15, "deterministic": 16,
 }
 # speck_kernel_kind_t (kernel id = kind * 16 + configuration)
 KERNEL_KINDS = {1: "analysis", 2: "binning", 3: "scan", 4: "sym_warp", 5: "sym_block", 6: "num_tiny", 7: "num_warp",
@@ -33,7 +33,7 @@ KERNEL_KINDS = {1: "analysis", 2: "binning", 3: "scan", 4: "sym_warp", 5: "sym_b
 PATHS = ["sym_warp", "sym_block_hash", "sym_merged", "sym_dense", "sym_dense_multi", "num_tiny", "num_warp_ordered",
          "num_warp_sorted", "num_block_ordered", "num_block_sorted", "num_merged", "num_dense", "num_dense_multi",
          "num_direct", "seg_hash", "seg_dense", "seg_windows", "long_bitmap", "long_bitmap_split", "sym_esc", "num_esc",
-         "num_esc_dup", "esc_fallback"]
+         "num_esc_dup", "esc_fallback", "num_det"]
 PATH_COUNT = 24
 # bin categories of speck_stats_t.bin_* (per pass)
 CATEGORIES = ["empty", "direct", "cfg0", "cfg1", "cfg2", "cfg3", "cfg4", "long", "tiny", "unused"]

@@ -113,3 +113,53 @@ def test_broadcast_protocol_gloo():
     assert res[0][1:3] == res[1][1:3]
     for a, b in zip(res[0][3:], res[1][3:]):
         assert np.array_equal(a, b)
+
+
+def _grid_worker(rank, world, port, q, pr, pc):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        A = W.rmat(10, 16, seed=9, dtype=torch.float64)
+        i, j = sdist.grid_coords(rank, pc)
+        groups = [dist.new_group([ii * pc + jj for jj in range(pc)]) for ii in range(pr)]
+        prods = torch.from_numpy(oracle.row_analysis(A, A)[0])
+        rb = sdist.partition_rows(prods, pr)
+        cb = sdist.column_bounds(A.cols, pc)
+        A_i = sdist.row_slice(A, rb[i], rb[i + 1])
+        B_j = sdist.column_block(A, cb[j], cb[j + 1])
+        tile = sdist.spgemm_2d_tile(A_i, B_j, local=_oracle_local)
+        Ci = sdist.assemble_row_block(tile, cb[j], groups[i], A.cols)
+        q.put((rank, rb[i], rb[i + 1], int(B_j.col.numel()), A.nnz, Ci.row_ptr.numpy(), Ci.col.numpy(), Ci.val.numpy()))
+    except Exception as e:
+        q.put((rank, repr(e)))
+        raise
+    finally:
+        dist.destroy_process_group()
+
+
+def test_2d_grid_without_b_replication():
+    """2 x 2 grid (SURVEY §8(f4)): rank (i, j) holds A's row block i and B's column block j only;
+    the tiles C_ij assembled per row block equal the oracle's rows, and no rank stores more than
+    ~half of B."""
+    world, pr, pc = 4, 2, 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_grid_worker, args=(r, world, port, q, pr, pc)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = {}
+    for _ in range(world):
+        item = q.get(timeout=300)
+        assert len(item) > 2, f"rank {item[0]} failed: {item[1]}"
+        res[item[0]] = item
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    A = W.rmat(10, 16, seed=9, dtype=torch.float64)
+    rp, col, val, _ = oracle.spgemm(A, A)
+    for r, (_, r0, r1, bnnz, annz, crp, ccol, cval) in res.items():
+        assert bnnz < 0.75 * annz                       # B is partitioned, not replicated
+        assert np.array_equal(crp, rp[r0:r1 + 1] - rp[r0])
+        assert np.array_equal(ccol, col[rp[r0]:rp[r1]])
+        assert np.allclose(cval, val[rp[r0]:rp[r1]], rtol=1e-12, atol=0)

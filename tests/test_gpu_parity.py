@@ -172,6 +172,12 @@ PATHS = [
     dict(disable_direct=1),
     dict(bucket_sort=0),
     dict(bucket_sort=1),
+    dict(bucket_sort=2),
+    dict(bucket_sort=0, fixed_group_size=1),
+    dict(bucket_sort=0, fixed_group_size=32),
+    dict(bucket_sort=0, fixed_group_size=1024),
+    dict(bucket_sort=0, fixed_group_size=-1),
+    dict(bucket_sort=0, fixed_group_size=-1, warp_rows=0),
     dict(concurrent_streams=1),
     dict(warp_rows=0),
     dict(warp_rows=0, global_lb_symbolic=0, global_lb_numeric=0),
@@ -462,7 +468,7 @@ def _path_inputs():
     As = W.random_sparse(4, 2000, 0.9, seed=33, dtype=torch.float32)
     out.append(("seg_hash", As, Bs, {}))
     # uniform short rows: merged blocks (Alg. 2) and the warp-per-row ordered map
-    U = W.random_sparse(3000, 3000, 0.012, seed=21, dtype=torch.float32)
+    U = W.random_sparse(3000, 3000, 0.006, seed=21, dtype=torch.float32)   # ~18 NZ/row: C rows of ~300
     out.append(("merged_numeric", U, None, dict(warp_rows=0, global_lb_symbolic=1, global_lb_numeric=1)))
     out.append(("warp_ordered", U, None, dict(bucket_sort=0, global_lb_symbolic=1, global_lb_numeric=1)))
     nb, lb = 3000, 1000
@@ -473,8 +479,9 @@ def _path_inputs():
     ac = np.concatenate([np.sort(rng.choice(nb, 24, replace=False)) for _ in range(700)])
     Am = W.csr_from_coo(700, nb, torch.tensor(ar), torch.tensor(ac), None, dtype=torch.float32, seed=19)
     out.append(("bitmap", Am, Bm, {}))
-    Av = W.csr_from_coo(4, nb, torch.arange(4).repeat_interleave(2000),
-                        torch.tensor(np.concatenate([np.sort(rng.choice(nb, 2000, replace=False)) for _ in range(4)])),
+    # 10 rows of 2M products (> 2^19: split over CTAs; 10 kept bitmaps of 128 KB fill the >= 1 MB pool)
+    Av = W.csr_from_coo(10, nb, torch.arange(10).repeat_interleave(2000),
+                        torch.tensor(np.concatenate([np.sort(rng.choice(nb, 2000, replace=False)) for _ in range(10)])),
                         None, dtype=torch.float32, seed=20)
     out.append(("bitmap_split", Av, Bm, dict(long_bitmap=2)))
     return out
@@ -502,6 +509,42 @@ def test_every_path_is_hit_and_correct(dev):
 # (seg_windows: a "windows" job needs >= 4 long rows per SM whose column range is too wide for the
 # bitmap CTA and whose window overhead beats segmenting — C5-sized inputs only)
 OPTIONAL_PATHS = {"num_warp_sorted", "esc_fallback", "seg_windows"}
+
+
+# ----------------------------------------------------------------------- deterministic mode (§8 f4)
+def _det_inputs():
+    yield "rmat_f32", W.rmat(12, 16, seed=81, dtype=torch.float32), None
+    yield "rmat_f64", W.rmat(11, 16, seed=82, dtype=torch.float64), None
+    # rows beyond the warp region (k_det_rows: ordered map) and beyond its map (dense windows)
+    yield "long_f32", W.random_sparse(40, 2000, 0.3, seed=83, dtype=torch.float32), \
+        W.random_sparse(2000, 120_000, 0.004, seed=84, dtype=torch.float32)
+    yield "cancel_f64", W.random_sparse(300, 300, 0.05, seed=85, dtype=torch.float64, zero_frac=0.2), None
+
+
+@pytest.mark.parametrize("warp_rows", [1, 0])
+def test_deterministic_mode_bit_exact_sequential(dev, warp_rows):
+    """SPECK_OPT_DETERMINISTIC: values equal, bit for bit, the oracle's left-to-right sum in the
+    inputs' precision (oracle_numeric_sequential, reading R15) on every row, and two runs agree
+    bit for bit; row_ptr / col_idx as always."""
+    for name, A, B in _det_inputs():
+        B = A if B is None else B
+        outs = []
+        for _ in range(2):
+            h = sp.Handle(0, deterministic=1, warp_rows=warp_rows, path_counters=1)
+            C = h.spgemm(A.to(dev), B.to(dev))
+            torch.cuda.synchronize()
+            outs.append((C, h.stats()["paths"]))
+            h.close()
+        (C, paths), (C2, _) = outs
+        rp, col, val = oracle.spgemm_sequential(A, B)
+        assert np.array_equal(C.row_ptr.cpu().numpy(), rp), name
+        assert np.array_equal(C.col.cpu().numpy(), col), name
+        g = C.val.cpu().numpy().astype(np.float64)
+        bad = np.nonzero(g != val)[0]
+        assert bad.size == 0, f"{name}: {bad.size} values differ from the sequential sum, first {bad[:5]}"
+        assert torch.equal(C.val, C2.val), name
+        if name == "long_f32":
+            assert paths["num_det"] > 0
 
 
 # ----------------------------------------------------------------------- transpose (§8 f2)

@@ -431,3 +431,37 @@ def test_compare_nan_even_with_huge_tolerance():
     rp, col, val, scale = _cmp_case()
     g = val.copy(); g[0] = np.nan
     assert not oracle.compare(rp, col, g, rp, col, val, scale, 1e300)["ok"]
+
+
+# ----------------------------------------------------------------- sequential (deterministic) values
+def test_sequential_sum_order_and_precision_pin():
+    """oracle.spgemm_sequential adds left to right in the inputs' precision (reading R15): for
+    fp32, 1e8 + 1 - 1e8 in that order is 0 (1e8 + 1 rounds to 1e8 in float), 1 in exact
+    arithmetic; reordered as 1e8 - 1e8 + 1 it is 1.  fp64 keeps the 1 (53-bit significand)."""
+    for dt, want in ((torch.float32, 0.0), (torch.float64, 1.0)):
+        A = W.CSR(1, 3, torch.tensor([0, 3]), torch.tensor([0, 1, 2], dtype=torch.int32), torch.ones(3, dtype=dt))
+        B = W.CSR(3, 2, torch.tensor([0, 1, 2, 3]), torch.tensor([1, 1, 1], dtype=torch.int32),
+                  torch.tensor([1e8, 1.0, -1e8], dtype=dt))
+        rp, col, val = oracle.spgemm_sequential(A, B)
+        assert col.tolist() == [1] and val.tolist() == [want]
+        B2 = W.CSR(3, 2, torch.tensor([0, 1, 2, 3]), torch.tensor([1, 1, 1], dtype=torch.int32),
+                   torch.tensor([1e8, -1e8, 1.0], dtype=dt))
+        assert oracle.spgemm_sequential(A, B2)[2].tolist() == [1.0]
+        # the exact oracle keeps the 1 either way
+        assert oracle.spgemm(A, B)[2].tolist() == [1.0]
+
+
+def test_sequential_equals_exact_on_integer_values():
+    """With small-integer values every order gives the exact result (C1 closed form)."""
+    A = W.poisson2d(32)
+    rp, col, val = oracle.spgemm_sequential(A, A)
+    rp2, col2, val2, _ = oracle.spgemm(A, A)
+    assert np.array_equal(rp, rp2) and np.array_equal(col, col2) and np.array_equal(val, val2)
+    # single product per entry (diagonal scaling): fl(a*b) exactly
+    D = W.CSR(50, 50, torch.arange(51), torch.arange(50, dtype=torch.int32), torch.linspace(0.1, 5, 50, dtype=torch.float32))
+    B = W.random_sparse(50, 40, 0.2, seed=9, dtype=torch.float32)
+    _, _, v = oracle.spgemm_sequential(D, B)
+    Bd = B.val.numpy()
+    want = np.concatenate([(np.float32(D.val[i].item()) * Bd[B.row_ptr[i]:B.row_ptr[i + 1]]).astype(np.float32)
+                           for i in range(50)])
+    assert np.array_equal(v, want.astype(np.float64))
