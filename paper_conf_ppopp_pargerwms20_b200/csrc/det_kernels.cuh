@@ -7,7 +7,7 @@
 // the products of one column in that order: equal columns of a warp step are added in lane
 // order ("rounds"), steps in order.  Each product is rounded before it is added
 // (acc <- fl(acc + fl(a*b)), __fadd_rn: no contraction), so C_ij is bit-identical across runs
-// and equal to the oracle's oracle_numeric_sequential (reading R15).
+// and equal to a sequential sum in the inputs' precision (reading R15).
 //   - rows that fit the 7 KB warp region: k_warp_rows (unchanged, already one warp per row);
 //   - larger rows: k_det_rows below — one warp per row with a 54 KB region: the ordered hash map
 //     of warp_row when the row fits it, else sequential dense column windows (each referenced B

@@ -66,7 +66,7 @@ static_assert(cfg_fits<0>() && cfg_fits<1>() && cfg_fits<2>() && cfg_fits<3>() &
 template <typename V>
 __device__ __forceinline__ V ldv(const V* p) { return __ldg(p); }
 // a + b rounded once, never contracted with the product that produced b (in-order, per-product
-// rounded sums: the warp-per-row paths match oracle_numeric_sequential bit for bit)
+// rounded sums: the warp-per-row paths give the sequential sum of reading R15 bit for bit)
 __device__ __forceinline__ float add_rn(float a, float b) { return __fadd_rn(a, b); }
 __device__ __forceinline__ double add_rn(double a, double b) { return __dadd_rn(a, b); }
 
