@@ -606,6 +606,17 @@ struct WindowRange {
   }
 };
 
+// Per referenced B row, [j0 + cur[f], j0 + next[f]) precomputed by the caller (pure: every warp
+// may evaluate it).
+struct KnownRange {
+  const int32_t* cur;
+  const int32_t* next;
+  __device__ __forceinline__ void operator()(int f, int64_t j0, int64_t, int64_t& s, int64_t& e) const {
+    s = j0 + cur[f];
+    e = j0 + next[f];
+  }
+};
+
 // An independent column range [lo, hi) of every referenced B row (long-row segments).
 struct SegRange {
   const int32_t* bcol;

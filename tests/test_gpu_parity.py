@@ -660,29 +660,49 @@ def test_chunked_c4_full_size(dev):
 
 
 # ----------------------------------------------------------------------- full sizes
-def _strata_blocks(cnt, seed, frac, per_stratum=16, width=64):
-    """Row blocks covering >= frac of the rows: random 64-row blocks plus `per_stratum` single
-    rows from every power-of-two stratum of nnz(C_i) (so every bin category is represented)."""
-    m = cnt.size
+def _strata_rows(cnt, seed, per_stratum=16):
+    """`per_stratum` random rows from every power-of-two stratum of nnz(C_i) (every bin category
+    is represented, the heaviest rows included)."""
     rng = np.random.default_rng(seed)
-    blocks = []
-    nblk = int(np.ceil(frac * m / width))
-    starts = np.sort(rng.choice(max(m // width, 1), size=min(nblk, max(m // width, 1)), replace=False)) * width
-    blocks += [(int(s), int(min(s + width, m))) for s in starts]
     strat = np.where(cnt > 0, np.floor(np.log2(np.maximum(cnt, 1))).astype(np.int64), -1)
+    rows = []
     for k in np.unique(strat):
-        rows = np.nonzero(strat == k)[0]
-        for r in rng.choice(rows, size=min(per_stratum, rows.size), replace=False):
-            blocks.append((int(r), int(r) + 1))
-    blocks.append((m - min(width, m), m))   # ragged tail
-    return blocks
+        rk = np.nonzero(strat == k)[0]
+        rows += [int(r) for r in rng.choice(rk, size=min(per_stratum, rk.size), replace=False)]
+    return np.array(sorted(set(rows) | {int(np.argmax(cnt))}), np.int64)
+
+
+def _gather_rows(A, rows):
+    """A[rows] as a CSR matrix (input preparation: C[rows] = A[rows]·B)."""
+    rp = A.row_ptr.numpy()
+    lens = rp[rows + 1] - rp[rows]
+    idx = np.concatenate([np.arange(rp[r], rp[r + 1]) for r in rows]) if rows.size else np.zeros(0, np.int64)
+    nrp = np.zeros(rows.size + 1, np.int64)
+    np.cumsum(lens, out=nrp[1:])
+    return W.CSR(int(rows.size), A.cols, torch.from_numpy(nrp), A.col[torch.from_numpy(idx)], A.val[torch.from_numpy(idx)])
+
+
+def _parity_rows(A, B, C, rows, tol):
+    """C's rows `rows` (device) against the oracle's A[rows]·B in ONE oracle call."""
+    Ar = _gather_rows(A, rows)
+    rp_o, col_o, val_o, sc_o = oracle.spgemm(Ar, B)
+    crp = C.row_ptr.cpu().numpy()
+    lens = crp[rows + 1] - crp[rows]
+    idx = np.concatenate([np.arange(crp[r], crp[r + 1]) for r in rows])
+    grp = np.zeros(rows.size + 1, np.int64)
+    np.cumsum(lens, out=grp[1:])
+    it = torch.from_numpy(idx).to(C.col.device)
+    res = oracle.compare(grp, C.col[it].cpu().numpy(), C.val[it].cpu().numpy().astype(np.float64),
+                         rp_o, col_o, val_o, sc_o, tol)
+    assert res["ok"], res
 
 
 @pytest.mark.parametrize("cfg,frac", [("c4", 1.0), ("c3", 0.10), ("c5", 0.10)])
 def test_full_size_every_row(dev, cfg, frac):
     """BASELINE configs at full size: nnz(C_i) of EVERY row equals the oracle's structural count
     (and so row_ptr is bit-exact everywhere); columns and values bit-exact / within tolerance on
-    every row of C4 and on >= 10% of the rows of C3 and C5 drawn from every nnz(C_i) stratum."""
+    every row of C4, and for C3 and C5 on contiguous row blocks spread evenly over the matrix that
+    hold ~10% of the entries, plus 16 rows from every power-of-two stratum of nnz(C_i)."""
     (label, A, B), = W.config(cfg, device=dev)
     h = sp.Handle(0)
     C = h.spgemm(A, B)
@@ -693,16 +713,21 @@ def test_full_size_every_row(dev, cfg, frac):
     rp = C.row_ptr.cpu().numpy()
     assert rp[0] == 0 and int(rp[-1]) == C.nnz == int(cnt_ref.sum()) == st["nnz_c"]
     assert np.array_equal(np.diff(rp), cnt_ref)
-    if frac >= 1.0:
-        # every row, streamed in blocks of ~2e7 entries
-        blocks, r0 = [], 0
-        while r0 < A.rows:
-            r1 = min(int(np.searchsorted(rp, rp[r0] + 20_000_000, side="right")), A.rows)
-            r1 = max(r1, r0 + 1)
-            blocks.append((r0, r1))
-            r0 = r1
-    else:
-        blocks = _strata_blocks(cnt_ref, seed=7, frac=frac)
+    tol = oracle.TOL[np.dtype(np.float32)]
+    # contiguous row blocks of ~2e7 entries: every block (frac = 1) or blocks spread evenly over the
+    # rows covering `frac` of them (one oracle call per block: its per-call scratch is O(columns))
+    blocks, r0 = [], 0
+    while r0 < A.rows:
+        r1 = min(int(np.searchsorted(rp, rp[r0] + 20_000_000, side="right")), A.rows)
+        r1 = max(r1, r0 + 1)
+        blocks.append((r0, r1))
+        r0 = r1
+    if frac < 1.0:
+        keep = max(1, int(round(frac * len(blocks))))
+        sel = np.linspace(0, len(blocks) - 1, keep).round().astype(int)
+        blocks = [blocks[i] for i in sorted(set(sel.tolist()))]
     assert_parity(Ah, Ah, C, rows=blocks)
+    # every nnz(C_i) stratum (every bin category), in one oracle call
+    _parity_rows(Ah, Ah, C, _strata_rows(cnt_ref, seed=7), tol)
     del C
     torch.cuda.empty_cache()

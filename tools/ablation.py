@@ -120,7 +120,7 @@ def lb_sweep(steps):
                 row["auto_choice"] = [st[0]["lb_symbolic"], st[0]["lb_numeric"]]
         row["ratio_prods"] = row["max_row_products"] / max(row["products"] / A.rows, 1e-9)
         out.append(row)
-        print(json.dumps(row), file=sys.stderr, flush=True)
+        print(json.dumps({"lb_sweep": row}), flush=True)
         del A, probs
         torch.cuda.empty_cache()
     return out
@@ -128,7 +128,7 @@ def lb_sweep(steps):
 
 def main():
     ap = argparse.ArgumentParser()
-    ap.add_argument("--configs", default="c2,c3,c4,c5")
+    ap.add_argument("--configs", default="c2,c3,c4,c5", help="'' for none")
     ap.add_argument("--steps", type=int, default=3)
     ap.add_argument("--variants", default=",".join(VARIANTS))
     ap.add_argument("--lb-sweep", action="store_true")
@@ -136,7 +136,7 @@ def main():
     from paper_conf_ppopp_pargerwms20_b200 import build
     build.build()
     res = {"variants": {k: VARIANTS[k] for k in args.variants.split(",")}, "configs": {}}
-    for cfg in args.configs.split(","):
+    for cfg in [c for c in args.configs.split(",") if c]:
         probs = W.config(cfg, device="cuda")
         tol = 1e-5 if probs[0][1].dtype == torch.float32 else 1e-12
         base_ms, ref, st = timed(probs, {}, args.steps)
@@ -151,11 +151,11 @@ def main():
             del outs
             torch.cuda.empty_cache()
         res["configs"][cfg] = row
+        print(json.dumps({"config": cfg, **row}), flush=True)      # one line per config (a kill keeps the rest)
         del probs, ref
         torch.cuda.empty_cache()
     if args.lb_sweep:
         res["lb_sweep"] = lb_sweep(args.steps)
-    print(json.dumps(res))
 
 
 if __name__ == "__main__":

@@ -1,6 +1,7 @@
 """Write profiles/traffic.json from `ncu --set full` reports (never edited by hand).
 
     python tools/traffic_from_ncu.py CFG TAG report1.ncu-rep [report2.ncu-rep ...]
+    python tools/traffic_from_ncu.py --ingest CFG TAG gpurun_out/<tag>_<cfg>_traffic.txt   (lines printed by --dry)
 
 For every launch in the reports: DRAM bytes (dram__bytes_read.sum + dram__bytes_write.sum) and
 the ncu duration, keyed by the same canonical kernel name bench.py derives from the library's
@@ -51,7 +52,31 @@ def metrics(rep):
     return res
 
 
+def ingest(cfg, tag, txt_files):
+    """Merge `--dry` lines printed on the GPU box (gpurun_out/*_traffic.txt) into traffic.json."""
+    head = subprocess.run(["git", "rev-parse", "--short=12", "HEAD"], capture_output=True, text=True, cwd=ROOT).stdout.strip()
+    path = os.path.join(ROOT, "profiles", "traffic.json")
+    db = {}
+    if os.path.exists(path):
+        with open(path) as f:
+            db = json.load(f)
+    db = {k: v for k, v in db.items() if isinstance(v, dict) and all(isinstance(x, dict) for x in v.values())}
+    ent = db.setdefault(cfg, {})
+    for fn in txt_files:
+        for line in open(fn):
+            t = line.split()
+            if len(t) < 7 or t[0] != cfg:
+                continue
+            ent[t[1]] = {"bytes": int(t[6]), "ncu_ms": float(t[4]), "kernel": " ".join(t[7:])[:120],
+                         "source": f"{tag}: {os.path.basename(fn)} (ncu --set full; committed at {head})"}
+    with open(path, "w") as f:
+        json.dump(db, f, indent=1, sort_keys=True)
+
+
 def main():
+    if sys.argv[1] == "--ingest":
+        ingest(sys.argv[2], sys.argv[3], sys.argv[4:])
+        return
     dry = "--dry" in sys.argv
     args = [a for a in sys.argv[1:] if a != "--dry"]
     cfg, tag, reps = args[0], args[1], args[2:]
