@@ -45,11 +45,18 @@ template <typename V>
 __host__ __device__ inline int64_t esc_capacity(int pass, int64_t bytes) {
   return (bytes - 320) * kEscLambda / ((int64_t)esc_entry_bytes<V>(pass) * kEscLambda + 8);
 }
-// rank of k among keys[s, en) (keys < k), two keys per iteration
+// rank of k among keys[s, en) (keys < k).  The trip count is the warp's largest bucket (a
+// warp-uniform loop: no divergent exits, no reconvergence barriers), 4 keys per iteration;
+// lanes past their bucket's end read nothing.  Inactive lanes pass s == en.
 __device__ __forceinline__ int esc_rank(const uint32_t* keys, int s, int en, uint32_t k) {
-  int r = 0, j = s;
-  for (; j + 2 <= en; j += 2) r += (keys[j] < k) + (keys[j + 1] < k);
-  if (j < en) r += keys[j] < k;
+  const int len = en - s;
+  const int mx = (int)__reduce_max_sync(0xffffffffu, (unsigned)len);
+  int r = 0;
+  for (int d = 0; d < mx; d += 4) {
+#pragma unroll
+    for (int u = 0; u < 4; ++u)
+      if (d + u < len) r += keys[s + d + u] < k;
+  }
   return r;
 }
 
@@ -256,13 +263,17 @@ __device__ __forceinline__ int esc_row(const SpgemmArgs<V>& p, unsigned char* re
   }
   if (n == cnt) {
     // no repeated column in the row: sorted position = bucket start + rank in the bucket
-    for (int e = t; e < n; e += T) {
-      const uint32_t k = keys[e];
+    for (int e0 = wi * 32; e0 < n; e0 += T) {          // warp-uniform: every lane calls esc_rank
+      const int e = e0 + lane;
+      const bool act = e < n;
+      const uint32_t k = act ? keys[e] : 0u;
       const uint32_t b = home(k);
-      const int s = b ? bc[b - 1] : 0, en = bc[b];
+      const int s = act ? (b ? bc[b - 1] : 0) : 0, en = act ? bc[b] : 0;
       const int r = esc_rank(keys, s, en, k);
-      p.C_col[cbase + s + r] = (int32_t)k;
-      p.C_val[cbase + s + r] = vals[e];
+      if (act) {
+        p.C_col[cbase + s + r] = (int32_t)k;
+        p.C_val[cbase + s + r] = vals[e];
+      }
     }
     esc_sync<NW>();
     return cnt;
@@ -296,15 +307,18 @@ __device__ __forceinline__ int esc_row(const SpgemmArgs<V>& p, unsigned char* re
   esc_sync<NW>();
   esc_scan<NW>(dc, NB, wi, red);      // dc[b] = first distinct position of bucket b
   // ---- W2: rank the surviving entries among the surviving entries of their bucket ------------
-  for (int e = t; e < n; e += T) {
-    const uint32_t k = keys[e];
-    if (k & kEscDropBit) continue;
-    const uint32_t b = home(k);
-    const int s = b ? bc[b - 1] : 0, en = bc[b];
-    const int r = esc_rank(keys, s, en, k);          // dropped keys have the top bit set: never smaller
-    const int64_t o = cbase + dc[b] + r;
-    p.C_col[o] = (int32_t)k;
-    p.C_val[o] = vals[e];
+  for (int e0 = wi * 32; e0 < n; e0 += T) {
+    const int e = e0 + lane;
+    const uint32_t kk = e < n ? keys[e] : kEscDropBit;
+    const bool act = !(kk & kEscDropBit);
+    const uint32_t b = act ? home(kk) : 0u;
+    const int s = act ? (b ? bc[b - 1] : 0) : 0, en = act ? bc[b] : 0;
+    const int r = esc_rank(keys, s, en, kk);          // dropped keys have the top bit set: never smaller
+    if (act) {
+      const int64_t o = cbase + dc[b] + r;
+      p.C_col[o] = (int32_t)kk;
+      p.C_val[o] = vals[e];
+    }
   }
   esc_sync<NW>();
   return cnt;

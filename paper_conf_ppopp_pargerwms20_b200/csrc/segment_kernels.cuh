@@ -256,36 +256,41 @@ __global__ void __launch_bounds__(kCfgThreads[kSegCfg], 1024 / kCfgThreads[kSegC
 
 // ------------------------------------------------------------------------------------
 // Long rows by bitmap + rank (B200 design for rows beyond the largest hash map whose column
-// range fits a shared-memory bitmap; C3's ~170k long rows): one CTA of 1024 threads per row.
+// range fits a shared-memory bitmap; C3's ~175k long rows): one CTA of 1024 threads per row.
 //   1. structure: every product sets its column's bit (the symbolic pass's dense bitmap,
 //      P:1064-1084) — or, when the symbolic step kept this row's bitmap in the pool
 //      (SPECK_OPT_BITMAP_REUSE), the bitmap is loaded from there and no product is expanded;
-//   2. one block scan gives every 1024-column group its output offset (gpre) and every 8-word
-//      sub-group its offset inside the group (spre); C.col is written in order from the bitmap
-//      (sorted by construction).  The position of column c in the row is
-//      gpre[group] + spre[sub-group] + popc(earlier words of the sub-group) + popc(bits below c);
-//   3. values, SLICED (round 2; rows with <= kSliceMaxNnzA NZ of A): the row's entries are cut
-//      into slices of consecutive groups that fit the rest of shared memory; per slice every
-//      product inside the slice's column range (each referenced B row resumes where the previous
-//      slice stopped) is added to its entry in shared memory, and the slice's C.val
-//      range is written once, coalesced.  (Round 1 zeroed C.val and added every product with a
-//      global RED.ADD.F32: 1.4e10 atomics for C3 at ~120 G/s, 1.7x C's bytes written to DRAM.)
-//      Rows with very long rows of A (C4: 200k NZ, where one sweep of the references per slice
-//      would cost as much as the products) keep the global atomics, as do rows split over
-//      several CTAs.
-// Hub rows of B (>= kLongB entries) referenced by a row are streamed by all 32 warps from a
-// shared list in the structure pass and the global-atomic value pass.  Columns are relative to
-// lo = colmin & ~31.
+//   2. one block scan gives every 32-bit word its exclusive prefix = the output position of
+//      its first entry; C.col is written in order from the bitmap (sorted by construction)
+//      and the row's C.val range is zeroed;
+//   3. values: every product's position is prefix[word] + popc(lower bits of its word), and
+//      a·b is added there with a global atomic (the row's C range stays in L2).
+// No column segments, no binary searches in B rows, no hash probing and no sort.  Hub rows of
+// B (>= kLongB entries) referenced by the row are streamed by all 32 warps from a shared list,
+// the other batches go round-robin over the warps, so no warp is left with a hub row alone.  Columns are
+// relative to lo = colmin & ~31; smem: bits (4 B/word) + per-word prefix within its 32-word
+// group (uint16) + per-group prefix (int32).
 // ------------------------------------------------------------------------------------
 constexpr int kBitmapThreads = 1024;
-// 140 B of shared memory per 1024-column group (128 bits + 4 group prefix + 8 sub-group prefixes),
-// and room for at least 4096 values of a slice
-constexpr int64_t kBitmapMaxCols = (int64_t)((kCfgMapBytes[kNumCfg - 1] - 4096 * 8 - 64) / 140) * 1024;
-constexpr int kSliceMaxNnzA = 8192;
+// 196 B of shared memory per 32-word group (128 bits + 4 prefix + 64 word prefixes)
+constexpr int64_t kBitmapMaxCols = (int64_t)(kCfgMapBytes[kNumCfg - 1] / 196) * 1024;
+
+// Split long rows (SegPlanArgs::split_max > 1) add their values with global atomics from several
+// CTAs: zero exactly those rows' C.val ranges first (one CTA per candidate; the rows that will
+// not be split zero their own range inside k_long_bitmap).
+template <typename V>
+__global__ void __launch_bounds__(256) k_zero_split_rows(const __grid_constant__ SpgemmArgs<V> p,
+                                                         const __grid_constant__ SegPlanArgs a) {
+  const int32_t row = a.cand[blockIdx.x];
+  if (row < p.row_lo || row >= p.row_hi) return;
+  const int64_t ob = a.C_rp[row], cnt = a.C_rp[row + 1] - ob;
+  if (cnt <= a.limit || !bitmap_row(a, row)) return;
+  if (a.bm_off[blockIdx.x] < 0 || p.prods[row] / kSplitProducts < 2) return;   // one piece: zeroed in place
+  for (int64_t i = threadIdx.x; i < cnt; i += blockDim.x) p.C_val[ob + i] = V(0);
+}
 
 template <typename V>
-__global__ void __launch_bounds__(kBitmapThreads, 1) k_long_bitmap(const __grid_constant__ SpgemmArgs<V> p,
-                                                                   const __grid_constant__ SegPlanArgs a) {
+__global__ void __launch_bounds__(kBitmapThreads, 1) k_long_bitmap(const __grid_constant__ SpgemmArgs<V> p, const __grid_constant__ SegPlanArgs a) {
   constexpr int T = kBitmapThreads, NW = T / 32;
   extern __shared__ __align__(16) unsigned char smem[];
   __shared__ int64_t part[NW + 1];
@@ -309,18 +314,14 @@ __global__ void __launch_bounds__(kBitmapThreads, 1) k_long_bitmap(const __grid_
   if (tid == 0) count_path(p.paths, pieces == 1 ? SPECK_PATH_LONG_BITMAP : SPECK_PATH_LONG_BITMAP_SPLIT);
   const uint32_t lo = (uint32_t)a.colmin[row] & ~31u;
   const int W = (int)(((int64_t)a.colmax[row] + 1 - lo + 31) / 32);
-  const int G = (W + 31) / 32;                                   // 1024-column groups
+  const int G = (W + 31) / 32;                                   // 32-word groups
   uint32_t* bits = reinterpret_cast<uint32_t*>(smem);
-  int32_t* gpre = reinterpret_cast<int32_t*>(smem + (size_t)G * 128);               // [G + 1]
-  uint16_t* spre = reinterpret_cast<uint16_t*>(smem + (size_t)G * 128 + (size_t)(G + 1) * 4);   // [4 G]
-  const size_t used = (((size_t)G * 128 + (size_t)(G + 1) * 4 + (size_t)G * 8) + 15) & ~(size_t)15;
-  V* sval = reinterpret_cast<V*>(smem + used);
-  const int vcap = (int)(((size_t)kCfgMapBytes[kNumCfg - 1] - used) / sizeof(V));
+  int32_t* gpre = reinterpret_cast<int32_t*>(smem + (size_t)G * 128);       // after 32*G words
+  uint16_t* wpre = reinterpret_cast<uint16_t*>(smem + (size_t)G * 128 + (size_t)G * 4);
   const int64_t ar0 = p.A_rp[row];
   const int arlen = (int)(p.A_rp[row + 1] - ar0);
   const int64_t a0 = ar0 + (int64_t)arlen * piece / pieces;             // this CTA's slice of A_i
   const int alen = (int)(ar0 + (int64_t)arlen * (piece + 1) / pieces - a0);
-  const bool sliced = pieces == 1 && arlen <= kSliceMaxNnzA;
   if (bmo >= 0) {
     // the symbolic step kept this row's bitmap: load it instead of rebuilding it (pass 1)
     const uint32_t* src = a.bm_pool + bmo;
@@ -329,11 +330,12 @@ __global__ void __launch_bounds__(kBitmapThreads, 1) k_long_bitmap(const __grid_
     for (int i = tid; i < G * 32; i += T) bits[i] = 0u;
   }
   // Rows whose referenced B rows are long on average (C3: ~800) rotate every chunk over all
-  // warps, each warp reading every batch (ALL mode); rows of A with many short references (C4:
-  // 200k NZ, ~20 products each) put hub rows of B (>= kLongB entries) in a shared list streamed
-  // by all warps, the other batches round-robin over the warps.
+  // warps, each warp reading every batch (ALL mode; the redundant batch loads are cheap next to
+  // the products).  Rows of A with many short references (C4: 200k NZ, ~20 products each) would
+  // pay 32x their A traffic that way: there hub rows of B (>= kLongB entries) go to a shared
+  // list streamed by all warps and the other batches go round-robin over the warps.
   bool listed = false;
-  if (!sliced && p.prods[row] < (int64_t)kAllAvgLen * arlen) listed = collect_long_rows<1, V>(p, a0, alen, longs);
+  if (p.prods[row] < (int64_t)kAllAvgLen * arlen) listed = collect_long_rows<1, V>(p, a0, alen, longs);
   else __syncthreads();
   // 1. structure
   auto set_bit = [&](uint32_t col, V, bool act) {
@@ -365,7 +367,7 @@ __global__ void __launch_bounds__(kBitmapThreads, 1) k_long_bitmap(const __grid_
     const int pc = __popc(word);
     const int incl = warp_incl_scan(pc);
     const int excl = incl - pc;
-    if ((lane & 7) == 0) spre[g * 4 + (lane >> 3)] = (uint16_t)excl;
+    wpre[g * 32 + lane] = (uint16_t)excl;
     if (lane == 0) gpre[g] = run;
     // C.col of the group: sparse groups per lane (a lane's entries are consecutive and the
     // group's entries span few sectors), dense groups one word at a time across the warp
@@ -392,73 +394,25 @@ __global__ void __launch_bounds__(kBitmapThreads, 1) k_long_bitmap(const __grid_
     }
     run += __shfl_sync(0xffffffffu, incl, 31);
   }
-  if (tid == 0) gpre[G] = (int32_t)cnt;
-  // position of column c (relative to lo) in the row
-  auto pos_of = [&](uint32_t c) {
-    const uint32_t w = c >> 5, g = w >> 5, sg = w >> 3;
-    int r = gpre[g] + (int)spre[sg] + __popc(bits[w] & ((1u << (c & 31)) - 1u));
-    for (uint32_t x = sg << 3; x < w; ++x) r += __popc(bits[x]);
-    return r;
-  };
-  if (!sliced) {
-    // 3. values, global atomics (split rows / very long rows of A): zero the row's values
-    // (coalesced) unless the host zeroed the split rows' range, then add every product
-    if (pieces == 1)
-      for (int64_t i = tid; i < cnt; i += T) p.C_val[ob + i] = V(0);
-    __syncthreads();
-    V* cv = p.C_val + ob;
-    auto add_val = [&](uint32_t col, V v, bool act) {
-      if (act) atomicAdd(cv + pos_of(col - lo), v);
-    };
-    if (listed) {
-      expand_long_list<1, V>(p, longs, wp, NW, add_val);
-      expand_row<1, V, true, false>(p, a0, alen, wp, NW, add_val, FullRange(), nullptr, kLongB);
-    } else {
-      expand_row<1, V, true, true>(p, a0, alen, wp, NW, add_val);
-    }
-    return;
-  }
-  // 3. values, sliced: slice s holds the groups whose first entry lies in [s*vc, (s+1)*vc),
-  // vc = vcap - 1024 (a group adds at most 1024 entries), so every slice fits shared memory
+  // zero the row's values (coalesced), then make the zeros visible to the block's atomics
+  // (split rows: C.val was zeroed before the launch)
+  if (pieces == 1)
+    for (int64_t i = tid; i < cnt; i += T) p.C_val[ob + i] = V(0);
   __syncthreads();
-  const unsigned slot = smid();
-  if (slot >= (unsigned)p.resume_slots) __trap();
-  int32_t* res = p.resume + (int64_t)slot * p.resume_stride;   // one CTA per SM (225 KB of shared memory)
-  int32_t* res_next = res + p.resume_stride / 2;
-  for (int f = tid; f < alen; f += T) res[f] = 0;
-  const int vc = vcap - 1024;
-  auto first_group = [&](int64_t x) {   // first group whose offset is >= x
-    int l = 0, h = G;
-    while (l < h) {
-      const int mid = (l + h) >> 1;
-      if (gpre[mid] < x) l = mid + 1; else h = mid;
+  // 3. values
+  V* cv = p.C_val + ob;
+  auto add_val = [&](uint32_t col, V v, bool act) {
+    if (act) {
+      const uint32_t c = col - lo, w = c >> 5;
+      const int r = gpre[w >> 5] + (int)wpre[w] + __popc(bits[w] & ((1u << (c & 31)) - 1u));
+      atomicAdd(cv + r, v);
     }
-    return l;
   };
-  const int nslices = (int)((cnt + vc - 1) / vc);
-  __syncthreads();
-  for (int sl = 0; sl < nslices; ++sl) {
-    const int gA = first_group((int64_t)sl * vc), gB = first_group((int64_t)(sl + 1) * vc);
-    if (gA >= gB) continue;
-    const int base = gpre[gA], n = gpre[gB] - base;
-    for (int i = tid; i < n; i += T) sval[i] = V(0);
-    __syncthreads();
-    const uint32_t whi = (uint32_t)min((int64_t)lo + (int64_t)gB * 1024, (int64_t)a.colmax[row] + 1);
-    // every referenced B row's part below whi: one binary search per reference, once per slice
-    // (the ALL-mode expansion below has every warp read every batch)
-    for (int f = tid; f < alen; f += T) {
-      const int32_t kc = p.A_col[a0 + f];
-      const int64_t j0 = p.B_rp[kc], j1 = p.B_rp[kc + 1];
-      res_next[f] = (int32_t)(lower_bound_col(p.B_col, j0 + res[f], j1, whi) - j0);
-    }
-    __syncthreads();
-    expand_row<1, V, true, true>(p, a0, alen, wp, NW, [&](uint32_t col, V v, bool act) {
-      if (act) atomicAdd(&sval[pos_of(col - lo) - base], v);
-    }, KnownRange{res, res_next});
-    __syncthreads();
-    { int32_t* t_ = res; res = res_next; res_next = t_; }
-    for (int i = tid; i < n; i += T) p.C_val[ob + base + i] = sval[i];
-    __syncthreads();
+  if (listed) {
+    expand_long_list<1, V>(p, longs, wp, NW, add_val);
+    expand_row<1, V, true, false>(p, a0, alen, wp, NW, add_val, FullRange(), nullptr, kLongB);
+  } else {
+    expand_row<1, V, true, true>(p, a0, alen, wp, NW, add_val);
   }
 }
 

@@ -283,6 +283,10 @@ speck_status_t set_smem_attrs(speck_handle_t h) {
   CK(cudaFuncSetAttribute(k_long_bitmap<V>, cudaFuncAttributeMaxDynamicSharedMemorySize, kCfgMapBytes[kNumCfg - 1]));
   CK(cudaFuncSetAttribute(k_warp_rows<0, V, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytesSym * (kWarpRowThreads / 32)));
   CK(cudaFuncSetAttribute(k_warp_rows<0, V, 3>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytesSym * (kWarpRowThreads / 32)));
+  CK(cudaFuncSetAttribute(k_warp_rows<0, V, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytesSym * (kWarpRowThreads / 32)));
+  CK(cudaFuncSetAttribute(k_warp_rows<1, V, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytes * (kWarpRowThreads / 32)));
+  CK(cudaFuncSetAttribute(k_warp_rows<1, V, 9>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytesTiny * (kWarpRowThreads / 32)));
+  CK(cudaFuncSetAttribute(k_warp_rows<1, V, 10>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytes * (kWarpRowThreads / 32)));
   CK(cudaFuncSetAttribute(k_warp_rows<1, V, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytes * (kWarpRowThreads / 32)));
   CK(cudaFuncSetAttribute(k_warp_rows<1, V, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytesTiny * (kWarpRowThreads / 32)));
   CK(cudaFuncSetAttribute(k_warp_rows<1, V, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytes * (kWarpRowThreads / 32)));
@@ -334,7 +338,12 @@ speck_status_t launch_warp_rows(speck_handle_t h, int pass, const SpgemmArgs<V>&
   const size_t smem = (size_t)wr_region_bytes(pass, md) * (kWarpRowThreads / 32);
   const int kt = kt_begin(h, s, pass == 0 ? SPECK_KERNEL_SYM_WARP : md == 1 ? SPECK_KERNEL_NUM_TINY : SPECK_KERNEL_NUM_WARP,
                           md, bin);
-  if (pass == 0 && a.esc >= 2) k_warp_rows<0, V, 3><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
+  if (a.fixed_g != 0) {   // the paper's grouped local load balancing (ablation instantiations)
+    if (pass == 0) k_warp_rows<0, V, 8><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
+    else if (mode == 1) k_warp_rows<1, V, 9><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
+    else if (mode == 2) k_warp_rows<1, V, 10><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
+    else k_warp_rows<1, V, 8><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
+  } else if (pass == 0 && a.esc >= 2) k_warp_rows<0, V, 3><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
   else if (pass == 0) k_warp_rows<0, V, 0><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
   else if (mode == 1) k_warp_rows<1, V, 1><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
   else if (mode == 2) k_warp_rows<1, V, 2><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
@@ -458,8 +467,7 @@ SegPlanArgs seg_plan_args(speck_handle_t h, const int64_t* C_rp) {
 // fixed groups of consecutive rows (LB off).
 template <typename V>
 speck_status_t run_pass(speck_handle_t h, int pass, int lb, const int64_t* cat_beg, const int64_t* cat_end,
-                        SpgemmArgs<V> a, int64_t need_max, const BinParams& bp, cudaStream_t s, int64_t c_off = 0,
-                        int64_t c_len = -1) {
+                        SpgemmArgs<V> a, int64_t need_max, const BinParams& bp, cudaStream_t s) {
   const int64_t m = a.m;
   if (!lb) {
     // no load balancing: one configuration with room for R rows of the longest size.
@@ -507,8 +515,9 @@ speck_status_t run_pass(speck_handle_t h, int pass, int lb, const int64_t* cat_b
     sa0 = seg_plan_args<V>(h, a.C_rp);
     if (sa0.bitmap_cols > 0 && sa0.bm_pool && h->n_cand <= kSplitMaxCand) {
       sa0.split_max = kSplitPieces;
-      // only this call's rows (the whole C, or a chunk's range of it)
-      CK(cudaMemsetAsync(a.C_val + c_off, 0, (size_t)(c_len < 0 ? h->nnz_c : c_len) * sizeof(V), s));
+      // zero the C.val ranges of the rows that will be split over several CTAs (only those)
+      k_zero_split_rows<V><<<(unsigned)h->n_cand, 256, 0, s>>>(a, sa0);
+      CKL();
     }
   }
   if ((st = fork(h, s, ns))) return st;
@@ -901,8 +910,7 @@ speck_status_t spgemm_rows_impl(speck_handle_t h, const speck_csr_t* A, const sp
   a.C_val = C_val - off;
   a.row_lo = r0;
   a.row_hi = r1;
-  const int64_t c_end = (int64_t)hp[2 * CAT_COUNT + 1];
-  return run_pass<V>(h, 1, 1, beg, end, a, h->max_cnt, bpn, s, off, c_end - off);
+  return run_pass<V>(h, 1, 1, beg, end, a, h->max_cnt, bpn, s);
 }
 
 // Device CSR transpose (transpose_kernels.cuh).

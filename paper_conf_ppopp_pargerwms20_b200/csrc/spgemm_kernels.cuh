@@ -815,7 +815,8 @@ __device__ __forceinline__ int warp_row(const SpgemmArgs<V>& p, uint32_t* rk, V*
   const uint64_t mmult = bkt_mult((uint32_t)(cmax - cmin + 1), S);
   // long rows use the order-preserving map (sorted write-out without a sort network);
   // short rows keep the scrambled hash (robust to clustered columns) and rank counting
-  const bool ordered = PASS == 1 && (MODE == 2 || (MODE == 0 && cnt > kSmallSeg));
+  constexpr int M = MODE & 7;
+  const bool ordered = PASS == 1 && (M == 2 || (M == 0 && cnt > kSmallSeg));
   int newc = 0, wrapped = 0;
   // 2 products per lane per chunk (fewer registers, more resident warps) for numeric MODE 1/2 rows
   // (C5 numeric 379 -> 362 ms, C2 tiny rows at 40 warps/SM 2.56 -> 2.35 ms) and symbolic rows
@@ -842,8 +843,9 @@ __device__ __forceinline__ int warp_row(const SpgemmArgs<V>& p, uint32_t* rk, V*
       }
     }
   };
-  if (p.fixed_g != 0) {
-    // the paper's local load balancing (Fig. 13 ablation): one warp = T threads, g per group
+  if (MODE & 8) {
+    // the paper's local load balancing (Fig. 13 ablation; own kernel instantiation, MODE | 8, so
+    // its registers do not weigh on the default path): one warp = T threads, g per group
     int g = p.fixed_g;
     if (g < 0) g = local_group_size(32, alen, warp_row_prods, warp_row_maxlen);
     expand_grouped<PASS, V>(p, a0, alen, 0, 1, g, ins);
@@ -856,12 +858,12 @@ __device__ __forceinline__ int warp_row(const SpgemmArgs<V>& p, uint32_t* rk, V*
     if (lane == 0) count_path(p.paths, SPECK_PATH_SYM_WARP);
     return warp_sum(newc);
   }
-  if (MODE != 1 && ordered && !__any_sync(0xffffffffu, wrapped)) {
+  if (M != 1 && ordered && !__any_sync(0xffffffffu, wrapped)) {
     // ordered map: every entry goes to (occupied slots before its run) + (rank in the run)
     if (lane == 0) count_path(p.paths, SPECK_PATH_NUM_WARP_ORDERED);
     warp_write_ordered<V>(rk, rv, S, 0u, S, cbase, 0, p.C_col, p.C_val);
   } else {
-    if (lane == 0) count_path(p.paths, MODE == 1 || cnt <= kSmallSeg ? SPECK_PATH_NUM_TINY : SPECK_PATH_NUM_WARP_SORTED);
+    if (lane == 0) count_path(p.paths, M == 1 || cnt <= kSmallSeg ? SPECK_PATH_NUM_TINY : SPECK_PATH_NUM_WARP_SORTED);
     warp_row_sorted_write<V>(rk, rv, S, cbase, p.C_col, p.C_val);
   }
   __syncwarp();
@@ -1248,18 +1250,21 @@ __device__ __noinline__ void dense_row(const SpgemmArgs<V>& p, BlockMeta& bm, in
 // load balancing, every row of A (p.rows == nullptr).
 // -----------------------------------------------------------------------------------
 template <int PASS, typename V, int MODE>
-__global__ void __launch_bounds__(kWarpRowThreads, wr_ctas_per_sm(PASS, MODE))
+__global__ void __launch_bounds__(kWarpRowThreads, wr_ctas_per_sm(PASS, MODE & 7))
     k_warp_rows(const __grid_constant__ SpgemmArgs<V> p, unsigned long long* __restrict__ counter) {
+  // MODE & 7: numeric 0 any row, 1 rows of <= kTinyCnt entries, 2 larger rows; symbolic 0 hash,
+  // 3 hash + bucket counting sort.  MODE & 8: the paper's grouped local load balancing (ablation).
   extern __shared__ __align__(16) unsigned char smem[];
   const int lane = lane_id();
-  constexpr int kRegion = wr_region_bytes(PASS, MODE);
+  constexpr int M = MODE & 7;
+  constexpr int kRegion = wr_region_bytes(PASS, M);
   unsigned char* region = smem + warp_id() * kRegion;
   uint32_t* rk = reinterpret_cast<uint32_t*>(region);
   V* rv = reinterpret_cast<V*>(region + (PASS == 0 ? 0u : wr_num_val_offset<V>(kRegion)));
   const uint32_t cap = PASS == 0 ? wr_sym_cap() : wr_num_cap<V>(kRegion);
   const int64_t esc_cap = esc_capacity<V>(PASS, kRegion);
   const int64_t n = p.n_entries;
-  constexpr bool kRange = (PASS == 1 && MODE != 1) || MODE == 3;
+  constexpr bool kRange = (PASS == 1 && M != 1) || M == 3;
   // row metadata, one field per lane: 0 A_rp[r], 1 A_rp[r+1], 2 prods[r] / C_rp[r], 3 C_rp[r+1],
   // 4 colmin[r], 5 colmax[r], 6 prods[r] (numeric) (one round trip instead of seven dependent loads)
   auto fetch = [&](int64_t e, int32_t& row, int64_t& mv) {
@@ -1273,8 +1278,8 @@ __global__ void __launch_bounds__(kWarpRowThreads, wr_ctas_per_sm(PASS, MODE))
       else if (lane == 3 && PASS == 1) mv = p.C_rp[row + 1];
       else if (lane == 4 && kRange) mv = p.colmin[row];   // column range: ordered maps only
       else if (lane == 5 && kRange) mv = p.colmax[row];
-      else if (lane == 6 && PASS == 1 && MODE != 1) mv = p.prods[row];
-      else if (lane == 7 && p.fixed_g < 0) mv = p.maxlen[row];     // dynamic g (paper's local LB)
+      else if (lane == 6 && PASS == 1 && M != 1) mv = p.prods[row];
+      else if (lane == 7 && (MODE & 8) && p.fixed_g < 0) mv = p.maxlen[row];   // dynamic g (paper's local LB)
     }
   };
   // rows are claimed kWarpRowChunk at a time (one same-address atomic per chunk: per-row
@@ -1349,7 +1354,7 @@ __global__ void __launch_bounds__(kWarpRowThreads, wr_ctas_per_sm(PASS, MODE))
     mv = mvn;
     fetch((int64_t)enn, rown, mvn);
     int c = -1;
-    if (MODE != 1 && (PASS == 1 || MODE == 3)) {
+    if (M != 1 && (PASS == 1 || M == 3) && !(MODE & 8)) {
       // rows whose products are (almost) all distinct columns: counting sort on column buckets
       // (esc_kernels.cuh); -1 = uneven buckets, the hash map below takes the row
       const int64_t np = PASS == 0 ? need : __shfl_sync(0xffffffffu, mv_prev6, 6);

@@ -460,6 +460,7 @@ def _path_inputs():
     A = W.random_sparse(6, 2000, 0.5, seed=31, dtype=torch.float32)
     B = W.random_sparse(2000, 200_000, 0.01, seed=32, dtype=torch.float32)
     out.append(("segments", A, B, {}))
+    out.append(("deterministic", A, B, dict(deterministic=1)))
     out.append(("windows", A, B, dict(segments=0)))
     # sparse long rows (~90k products over 2M columns): hashed column segments
     cols = np.sort(rng.choice(2_000_000, size=(2000, 50), replace=True), axis=1).astype(np.int64)
