@@ -856,6 +856,7 @@ __device__ __forceinline__ int warp_row(const SpgemmArgs<V>& p, uint32_t* rk, V*
   }
   if (PASS == 0) {
     if (lane == 0) count_path(p.paths, SPECK_PATH_SYM_WARP);
+    __syncwarp();   // the region's last probes complete before the next row clears it (racecheck)
     return warp_sum(newc);
   }
   if (M != 1 && ordered && !__any_sync(0xffffffffu, wrapped)) {
@@ -871,21 +872,19 @@ __device__ __forceinline__ int warp_row(const SpgemmArgs<V>& p, uint32_t* rk, V*
 }
 
 template <int CFG, int PASS, typename V>
-__device__ __noinline__ void dense_row(const SpgemmArgs<V>& p, BlockMeta& bm, int b0, unsigned char* smem, int* chist);
+__device__ __noinline__ void dense_row(const SpgemmArgs<V>& p, BlockMeta& bm, int b0, unsigned char* smem, int* chist,
+                                       int64_t gidx);
 
 // -----------------------------------------------------------------------------------
 // The per-configuration kernel.  PASS 0 = symbolic, 1 = numeric.
 // -----------------------------------------------------------------------------------
 template <int CFG, int PASS, typename V>
-__global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_spgemm(const __grid_constant__ SpgemmArgs<V> p) {
+__device__ __forceinline__ void spgemm_group(const SpgemmArgs<V>& p, const int64_t gidx, unsigned char* smem, BlockMeta& bm,
+                                             int* chist) {
   constexpr int T = kCfgThreads[CFG];
-  
-  extern __shared__ __align__(16) unsigned char smem[];
-  __shared__ BlockMeta bm;
-  __shared__ int chist[(CFG == kNumCfg - 1 && PASS == 0) ? kMaxChunks : 1];
   const int tid = threadIdx.x;
 
-  const int64_t e0 = (int64_t)blockIdx.x * p.group_rows;
+  const int64_t e0 = gidx * p.group_rows;
   const int ne = (int)(p.n_entries - e0 < p.group_rows ? p.n_entries - e0 : p.group_rows);
   if (ne <= 0) return;
 
@@ -1027,7 +1026,7 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
         if (PASS == 0 && tid == 0) p.cnt[bm.row[b0]] = c;
         if (chunks) {
           __syncthreads();
-          int32_t* dst = p.chunk_cnt + (int64_t)blockIdx.x * p.nchunks;
+          int32_t* dst = p.chunk_cnt + gidx * p.nchunks;
           for (int i = tid; i < p.nchunks; i += T) dst[i] = chist[i];
         }
       }
@@ -1116,7 +1115,7 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
             if (kk != kEmptyKey) atomicAdd(&chist[kk >> p.chunk_shift], 1);
           }
           __syncthreads();
-          int32_t* dst = p.chunk_cnt + (int64_t)blockIdx.x * p.nchunks;
+          int32_t* dst = p.chunk_cnt + gidx * p.nchunks;
           for (int i = tid; i < p.nchunks; i += T) dst[i] = chist[i];
         }
       } else if (!any_wrap) {
@@ -1130,10 +1129,41 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
         block_sorted_write<T, V>(keys, vals, capt, bm, p.C_col, p.C_val);
       }
     } else {
-      dense_row<CFG, PASS, V>(p, bm, b0, smem, chist);
+      dense_row<CFG, PASS, V>(p, bm, b0, smem, chist, gidx);
     }
     __syncthreads();
     b0 = b1;
+  }
+}
+
+// One CTA per group of entries (grid = groups).
+template <int CFG, int PASS, typename V>
+__global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_spgemm(const __grid_constant__ SpgemmArgs<V> p) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  __shared__ BlockMeta bm;
+  __shared__ int chist[(CFG == kNumCfg - 1 && PASS == 0) ? kMaxChunks : 1];
+  spgemm_group<CFG, PASS, V>(p, (int64_t)blockIdx.x, smem, bm, chist);
+}
+
+// Persistent CTAs (grid = SMs x resident CTAs): each pulls the next group from a counter, so
+// millions of single-row groups (C5: 4.3M rows in configuration 1) cost no CTA launches and a
+// CTA's barrier waits overlap the other resident CTAs' work.
+template <int CFG, int PASS, typename V>
+__global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG])
+    k_spgemm_persist(const __grid_constant__ SpgemmArgs<V> p, unsigned long long* __restrict__ counter) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  __shared__ BlockMeta bm;
+  __shared__ int chist[(CFG == kNumCfg - 1 && PASS == 0) ? kMaxChunks : 1];
+  __shared__ unsigned long long s_g;
+  const int64_t ngroups = (p.n_entries + p.group_rows - 1) / p.group_rows;
+  while (true) {
+    if (threadIdx.x == 0) s_g = atomicAdd(counter, 1ull);
+    __syncthreads();
+    const int64_t g = (int64_t)s_g;
+    __syncthreads();
+    if (g >= ngroups) break;
+    spgemm_group<CFG, PASS, V>(p, g, smem, bm, chist);
+    __syncthreads();
   }
 }
 
@@ -1141,7 +1171,8 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
 // Windows over [colmin, colmax] (Fig. 5); kept out of line so the hash paths'
 // hot loops stay compact in the instruction cache.
 template <int CFG, int PASS, typename V>
-__device__ __noinline__ void dense_row(const SpgemmArgs<V>& p, BlockMeta& bm, int b0, unsigned char* smem, int* chist) {
+__device__ __noinline__ void dense_row(const SpgemmArgs<V>& p, BlockMeta& bm, int b0, unsigned char* smem, int* chist,
+                                       int64_t gidx) {
   constexpr int T = kCfgThreads[CFG];
   constexpr int NW = T / 32;
   const int tid = threadIdx.x;
@@ -1223,7 +1254,7 @@ __device__ __noinline__ void dense_row(const SpgemmArgs<V>& p, BlockMeta& bm, in
           const unsigned long long need = ((unsigned long long)nwords + 3ull) & ~3ull;
           const unsigned long long o = atomicAdd(p.bm_ctr, need);
           s_bmo = o + need <= p.bm_pool_words ? (long long)o : -1ll;
-          p.bm_off[blockIdx.x] = s_bmo;
+          p.bm_off[gidx] = s_bmo;
         }
         __syncthreads();
         const long long o = s_bmo;
@@ -1233,7 +1264,7 @@ __device__ __noinline__ void dense_row(const SpgemmArgs<V>& p, BlockMeta& bm, in
         }
       }
       if (chunks) {
-        int32_t* dst = p.chunk_cnt + (int64_t)blockIdx.x * p.nchunks;
+        int32_t* dst = p.chunk_cnt + gidx * p.nchunks;
         for (int i = tid; i < p.nchunks; i += T) dst[i] = chist[i];
       }
     }

@@ -22,7 +22,8 @@ fi
 i=0
 IFS=";" read -ra KS <<< "${K:-}"
 for k in "${KS[@]}"; do
-  timeout 900 ncu --set full --clock-control none --import-source on -k "regex:$k" --kernel-name-base demangled -c 1 \
+  rm -f /tmp/rep/k$i.ncu-rep
+  timeout 900 ncu -f --set full --clock-control none --import-source on -k "regex:$k" --kernel-name-base demangled -c 1 \
     -o /tmp/rep/k$i python bench.py $B --steps 1 --warmup 3 > gpurun_out/${TAG}_${CFG}_k$i.log 2>&1
   python tools/ncu_summary.py /tmp/rep/k$i.ncu-rep 0 > gpurun_out/${TAG}_${CFG}_k$i.txt 2>&1
   python tools/ncu_sass.py /tmp/rep/k$i.ncu-rep 0 > gpurun_out/${TAG}_${CFG}_k${i}_sass.txt 2>&1
