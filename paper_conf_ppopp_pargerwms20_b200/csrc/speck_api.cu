@@ -260,44 +260,15 @@ void* spgemm_fn(int cfg, int pass) {
 }
 
 template <typename V>
-void* spgemm_persist_fn(int cfg, int pass) {
-  switch (cfg * 2 + pass) {
-    case 0: return (void*)k_spgemm_persist<0, 0, V>;
-    case 1: return (void*)k_spgemm_persist<0, 1, V>;
-    case 2: return (void*)k_spgemm_persist<1, 0, V>;
-    case 3: return (void*)k_spgemm_persist<1, 1, V>;
-    case 4: return (void*)k_spgemm_persist<2, 0, V>;
-    case 5: return (void*)k_spgemm_persist<2, 1, V>;
-    case 6: return (void*)k_spgemm_persist<3, 0, V>;
-    case 7: return (void*)k_spgemm_persist<3, 1, V>;
-    case 8: return (void*)k_spgemm_persist<4, 0, V>;
-    default: return (void*)k_spgemm_persist<4, 1, V>;
-  }
-}
-
-#ifndef SPECK_PERSIST
-#define SPECK_PERSIST 1
-#endif
-
-template <typename V>
 speck_status_t launch_spgemm(speck_handle_t h, int cfg, int pass, const SpgemmArgs<V>& a, cudaStream_t s, int bin) {
   if (a.n_entries <= 0) return SPECK_OK;
   const int64_t grid = (a.n_entries + a.group_rows - 1) / a.group_rows;
-  const int64_t resident = (int64_t)h->num_sms * (1024 / kCfgThreads[cfg]);
+  // (persistent CTAs pulling groups from a counter were tried: C5 336 -> 350 ms, the resident
+  // grid keeps the other bins' kernels from overlapping; one CTA per group it is)
   const int kt = kt_begin(h, s, pass == 0 ? SPECK_KERNEL_SYM_BLOCK : SPECK_KERNEL_NUM_BLOCK, cfg, bin);
-  if (SPECK_PERSIST && grid > 2 * resident) {
-    // many groups: persistent CTAs pulling groups from a counter (k_spgemm_persist)
-    unsigned long long* ctr =
-        reinterpret_cast<unsigned long long*>(static_cast<char*>(h->small.p) + 1536 + 8 * (cfg * 2 + pass));
-    CK(cudaMemsetAsync(ctr, 0, 8, s));
-    void* args[] = {(void*)&a, (void*)&ctr};
-    CK(cudaLaunchKernel(spgemm_persist_fn<V>(cfg, pass), dim3((unsigned)resident), dim3(kCfgThreads[cfg]), args,
-                        (size_t)kCfgMapBytes[cfg], s));
-  } else {
-    void* args[] = {(void*)&a};
-    CK(cudaLaunchKernel(spgemm_fn<V>(cfg, pass), dim3((unsigned)grid), dim3(kCfgThreads[cfg]), args,
-                        (size_t)kCfgMapBytes[cfg], s));
-  }
+  void* args[] = {(void*)&a};
+  CK(cudaLaunchKernel(spgemm_fn<V>(cfg, pass), dim3((unsigned)grid), dim3(kCfgThreads[cfg]), args,
+                      (size_t)kCfgMapBytes[cfg], s));
   kt_end(h, s, kt);
   ++h->launches;
   return SPECK_OK;
@@ -306,10 +277,8 @@ speck_status_t launch_spgemm(speck_handle_t h, int cfg, int pass, const SpgemmAr
 template <typename V>
 speck_status_t set_smem_attrs(speck_handle_t h) {
   for (int c = 0; c < kNumCfg; ++c)
-    for (int pass = 0; pass < 2; ++pass) {
+    for (int pass = 0; pass < 2; ++pass)
       CK(cudaFuncSetAttribute(spgemm_fn<V>(c, pass), cudaFuncAttributeMaxDynamicSharedMemorySize, kCfgMapBytes[c]));
-      CK(cudaFuncSetAttribute(spgemm_persist_fn<V>(c, pass), cudaFuncAttributeMaxDynamicSharedMemorySize, kCfgMapBytes[c]));
-    }
   CK(cudaFuncSetAttribute(k_segments<V>, cudaFuncAttributeMaxDynamicSharedMemorySize, kCfgMapBytes[kSegCfg]));
   CK(cudaFuncSetAttribute(k_tr_sort_block<V>, cudaFuncAttributeMaxDynamicSharedMemorySize, kTrSmemSort * (4 + (int)sizeof(V))));
   CK(cudaFuncSetAttribute(k_det_rows<V>, cudaFuncAttributeMaxDynamicSharedMemorySize, kDetRegion * kDetWarps));

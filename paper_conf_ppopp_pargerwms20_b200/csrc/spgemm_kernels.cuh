@@ -1145,28 +1145,6 @@ __global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG]) k_s
   spgemm_group<CFG, PASS, V>(p, (int64_t)blockIdx.x, smem, bm, chist);
 }
 
-// Persistent CTAs (grid = SMs x resident CTAs): each pulls the next group from a counter, so
-// millions of single-row groups (C5: 4.3M rows in configuration 1) cost no CTA launches and a
-// CTA's barrier waits overlap the other resident CTAs' work.
-template <int CFG, int PASS, typename V>
-__global__ void __launch_bounds__(kCfgThreads[CFG], 1024 / kCfgThreads[CFG])
-    k_spgemm_persist(const __grid_constant__ SpgemmArgs<V> p, unsigned long long* __restrict__ counter) {
-  extern __shared__ __align__(16) unsigned char smem[];
-  __shared__ BlockMeta bm;
-  __shared__ int chist[(CFG == kNumCfg - 1 && PASS == 0) ? kMaxChunks : 1];
-  __shared__ unsigned long long s_g;
-  const int64_t ngroups = (p.n_entries + p.group_rows - 1) / p.group_rows;
-  while (true) {
-    if (threadIdx.x == 0) s_g = atomicAdd(counter, 1ull);
-    __syncthreads();
-    const int64_t g = (int64_t)s_g;
-    __syncthreads();
-    if (g >= ngroups) break;
-    spgemm_group<CFG, PASS, V>(p, g, smem, bm, chist);
-    __syncthreads();
-  }
-}
-
 // ============================ DENSE ACCUMULATOR (single row) =============================
 // Windows over [colmin, colmax] (Fig. 5); kept out of line so the hash paths'
 // hot loops stay compact in the instruction cache.
