@@ -24,9 +24,17 @@
 namespace speck {
 
 // Table 2 thresholds: {ratio, rows} for all kernels and for the largest ones.
+// The paper's Titan V values were {39.2, 28000, 6.0, 5431} (symbolic) and {10.5, 23006, 1.3, 1238}
+// (numeric).  B200 re-tuning (tools/ablation.py --lb-sweep,
+// profiles/r02/r02r_ablation_c3_lbsweep.jsonl): on R-MAT families of scale 12-18 and uniform
+// matrices, global balancing wins from ~64k rows on at any skew above ~4 (scale 18, a = .35,
+// ratio 12: 8.33 ms off, 3.06 ms on — the Titan V threshold 39.2 left the symbolic step
+// unbalanced, 3.66 ms) and loses below ~16k rows (scale 12: 0.26 off vs 0.74 on: the binning
+// launches cost more than the imbalance), so both steps use {4.0, 32768}; rows that need the
+// largest configuration still force it on (long rows are only handled by the binned path).
 struct LbThresholds { double ratio, rows, ratio_big, rows_big; int big_from_cfg; };
-static const LbThresholds kLbSym = {39.2, 28000, 6.0, 5431, 2};  // "*" = three largest (caption, reading R11)
-static const LbThresholds kLbNum = {10.5, 23006, 1.3, 1238, 3};  // "*" = two largest
+static const LbThresholds kLbSym = {4.0, 32768, 4.0, 32768, 2};  // "*" = three largest (caption, reading R11)
+static const LbThresholds kLbNum = {4.0, 32768, 4.0, 32768, 3};  // "*" = two largest
 
 struct Buf {
   void* p = nullptr;
@@ -289,6 +297,9 @@ speck_status_t set_smem_attrs(speck_handle_t h) {
   CK(cudaFuncSetAttribute(k_warp_rows<1, V, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytes * (kWarpRowThreads / 32)));
   CK(cudaFuncSetAttribute(k_warp_rows<1, V, 9>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytesTiny * (kWarpRowThreads / 32)));
   CK(cudaFuncSetAttribute(k_warp_rows<1, V, 10>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytes * (kWarpRowThreads / 32)));
+  CK(cudaFuncSetAttribute(k_warp_rows<1, V, 16>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytes * (kWarpRowThreads / 32)));
+  CK(cudaFuncSetAttribute(k_warp_rows<1, V, 17>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytesTiny * (kWarpRowThreads / 32)));
+  CK(cudaFuncSetAttribute(k_warp_rows<1, V, 18>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytes * (kWarpRowThreads / 32)));
   CK(cudaFuncSetAttribute(k_warp_rows<1, V, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytes * (kWarpRowThreads / 32)));
   CK(cudaFuncSetAttribute(k_warp_rows<1, V, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytesTiny * (kWarpRowThreads / 32)));
   CK(cudaFuncSetAttribute(k_warp_rows<1, V, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytes * (kWarpRowThreads / 32)));
@@ -340,7 +351,11 @@ speck_status_t launch_warp_rows(speck_handle_t h, int pass, const SpgemmArgs<V>&
   const size_t smem = (size_t)wr_region_bytes(pass, md) * (kWarpRowThreads / 32);
   const int kt = kt_begin(h, s, pass == 0 ? SPECK_KERNEL_SYM_WARP : md == 1 ? SPECK_KERNEL_NUM_TINY : SPECK_KERNEL_NUM_WARP,
                           md, bin);
-  if (a.fixed_g != 0) {   // the paper's grouped local load balancing (ablation instantiations)
+  if (pass == 1 && a.det) {   // deterministic mode: in-order adds (own instantiations)
+    if (mode == 1) k_warp_rows<1, V, 17><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
+    else if (mode == 2) k_warp_rows<1, V, 18><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
+    else k_warp_rows<1, V, 16><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
+  } else if (a.fixed_g != 0) {   // the paper's grouped local load balancing (ablation instantiations)
     if (pass == 0) k_warp_rows<0, V, 8><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
     else if (mode == 1) k_warp_rows<1, V, 9><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
     else if (mode == 2) k_warp_rows<1, V, 10><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
@@ -424,6 +439,7 @@ SpgemmArgs<V> base_args(speck_handle_t h, const speck_csr_t* A, const speck_csr_
   a.fixed_g = (int)h->opt_fixed_g;
   a.esc = h->opt_det ? 0 : (int)h->opt_esc;          // deterministic: one warp per row, in-order adds
   if (h->opt_det) a.fixed_g = 0;
+  a.det = (int)h->opt_det;
   a.paths = h->opt_paths ? static_cast<unsigned long long*>(h->paths.p) : nullptr;
   a.row_lo = 0;
   a.row_hi = INT64_MAX;
