@@ -86,7 +86,7 @@ __global__ void __launch_bounds__(32 * kDetWarps, 1) k_det_rows(const __grid_con
       V* rv = reinterpret_cast<V*>(region + (((size_t)cap * 4 + 15) & ~(size_t)15));
       const uint64_t w32 = ((uint64_t)cnt * 5 / 2 + 31) & ~(uint64_t)31;
       const uint32_t S = (uint32_t)(w32 < 64 ? 64 : (w32 > cap ? cap : w32));
-      warp_row<1, V, 16>(p, rk, rv, S, a0, alen, cmn, cmx, cnt, cb);
+      warp_row<1, V, 0>(p, rk, rv, S, a0, alen, cmn, cmx, cnt, cb);
       continue;
     }
     // dense windows over [colmin, colmax], products of every window in the order of eq. (1)

@@ -297,9 +297,6 @@ speck_status_t set_smem_attrs(speck_handle_t h) {
   CK(cudaFuncSetAttribute(k_warp_rows<1, V, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytes * (kWarpRowThreads / 32)));
   CK(cudaFuncSetAttribute(k_warp_rows<1, V, 9>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytesTiny * (kWarpRowThreads / 32)));
   CK(cudaFuncSetAttribute(k_warp_rows<1, V, 10>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytes * (kWarpRowThreads / 32)));
-  CK(cudaFuncSetAttribute(k_warp_rows<1, V, 16>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytes * (kWarpRowThreads / 32)));
-  CK(cudaFuncSetAttribute(k_warp_rows<1, V, 17>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytesTiny * (kWarpRowThreads / 32)));
-  CK(cudaFuncSetAttribute(k_warp_rows<1, V, 18>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytes * (kWarpRowThreads / 32)));
   CK(cudaFuncSetAttribute(k_warp_rows<1, V, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytes * (kWarpRowThreads / 32)));
   CK(cudaFuncSetAttribute(k_warp_rows<1, V, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytesTiny * (kWarpRowThreads / 32)));
   CK(cudaFuncSetAttribute(k_warp_rows<1, V, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRegionBytes * (kWarpRowThreads / 32)));
@@ -351,11 +348,7 @@ speck_status_t launch_warp_rows(speck_handle_t h, int pass, const SpgemmArgs<V>&
   const size_t smem = (size_t)wr_region_bytes(pass, md) * (kWarpRowThreads / 32);
   const int kt = kt_begin(h, s, pass == 0 ? SPECK_KERNEL_SYM_WARP : md == 1 ? SPECK_KERNEL_NUM_TINY : SPECK_KERNEL_NUM_WARP,
                           md, bin);
-  if (pass == 1 && a.det) {   // deterministic mode: in-order adds (own instantiations)
-    if (mode == 1) k_warp_rows<1, V, 17><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
-    else if (mode == 2) k_warp_rows<1, V, 18><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
-    else k_warp_rows<1, V, 16><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
-  } else if (a.fixed_g != 0) {   // the paper's grouped local load balancing (ablation instantiations)
+  if (a.fixed_g != 0) {   // the paper's grouped local load balancing (ablation instantiations)
     if (pass == 0) k_warp_rows<0, V, 8><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
     else if (mode == 1) k_warp_rows<1, V, 9><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
     else if (mode == 2) k_warp_rows<1, V, 10><<<(unsigned)grid, kWarpRowThreads, smem, s>>>(a, ctr);
@@ -439,7 +432,6 @@ SpgemmArgs<V> base_args(speck_handle_t h, const speck_csr_t* A, const speck_csr_
   a.fixed_g = (int)h->opt_fixed_g;
   a.esc = h->opt_det ? 0 : (int)h->opt_esc;          // deterministic: one warp per row, in-order adds
   if (h->opt_det) a.fixed_g = 0;
-  a.det = (int)h->opt_det;
   a.paths = h->opt_paths ? static_cast<unsigned long long*>(h->paths.p) : nullptr;
   a.row_lo = 0;
   a.row_hi = INT64_MAX;

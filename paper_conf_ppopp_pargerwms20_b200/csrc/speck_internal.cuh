@@ -322,7 +322,6 @@ struct SpgemmArgs {
   int fixed_g;               // >0: fixed group size
   int esc;                   // bucket counting-sort rows (esc_kernels.cuh): 0 off, 1 numeric, 2 + symbolic
   unsigned long long* paths; // SPECK_OPT_PATH_COUNTERS: rows per speck_path_t (nullptr: off)
-  int det;                   // SPECK_OPT_DETERMINISTIC: in-order, per-product-rounded sums
   int64_t row_lo, row_hi;    // row-range numeric (speck_spgemm_rows): long-row jobs outside [row_lo, row_hi) exit
   // symbolic out
   int64_t* cnt;

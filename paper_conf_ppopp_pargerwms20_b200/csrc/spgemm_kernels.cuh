@@ -834,31 +834,14 @@ __device__ __forceinline__ int warp_row(const SpgemmArgs<V>& p, uint32_t* rk, V*
         s = ordered ? probe_insert_bkt(rk, S >> 3, bkt_home(col, mlo, mmult), col, &wrapped)
                     : probe_insert_mono(rk, S, hash_slot(col, S), col, &wrapped);
       }
-      if (MODE & 16) {
-        // deterministic mode (own instantiation, MODE | 16): equal keys of the step add in lane
-        // order, one round each
-        s = __shfl_sync(0xffffffffu, s, __ffs(peers) - 1);   // the key's slot, from its first lane
-        const int rank = __popc(peers & lt);
-        const int maxg = (int)__reduce_max_sync(0xffffffffu, (unsigned)__popc(peers));
-        for (int t = 0; t < maxg; ++t) {
-          if (act && rank == t) rv[s] = add_rn(rv[s], v);
-          __syncwarp();
-        }
-      } else {
-        // the first lane of each key (which claimed the slot) sums its peers' values in
-        // registers and adds once
-        const int maxg = (int)__reduce_max_sync(0xffffffffu, (unsigned)__popc(peers));
-        V sum = v;
-        if (maxg > 1) {
-          uint32_t others = (peers & lt) ? 0u : (peers & ~(1u << lane_id()));
-          for (int t = 1; t < maxg; ++t) {
-            int src = lane_id();
-            if (others) { src = __ffs(others) - 1; others &= others - 1; }
-            const V x = __shfl_sync(0xffffffffu, v, src);
-            if (src != lane_id()) sum += x;
-          }
-        }
-        if (act && !(peers & lt)) rv[s] += sum;
+      // equal keys of the warp step add in lane order, one round each: no atomics on values, and
+      // the in-order, per-product-rounded sum of reading R15 (summing the peers in registers
+      // first was tried: C2 numeric A*P 2.35 -> 2.52 ms, fp64 shuffles cost two instructions)
+      s = __shfl_sync(0xffffffffu, s, __ffs(peers) - 1);   // the key's slot, from its first lane
+      const int rank = __popc(peers & lt);
+      const int maxg = (int)__reduce_max_sync(0xffffffffu, (unsigned)__popc(peers));
+      for (int t = 0; t < maxg; ++t) {
+        if (act && rank == t) rv[s] = add_rn(rv[s], v);
         __syncwarp();
       }
     }
@@ -1283,7 +1266,6 @@ __global__ void __launch_bounds__(kWarpRowThreads, wr_ctas_per_sm(PASS, MODE & 7
     k_warp_rows(const __grid_constant__ SpgemmArgs<V> p, unsigned long long* __restrict__ counter) {
   // MODE & 7: numeric 0 any row, 1 rows of <= kTinyCnt entries, 2 larger rows; symbolic 0 hash,
   // 3 hash + bucket counting sort.  MODE & 8: the paper's grouped local load balancing (ablation).
-  // MODE & 16: deterministic mode (in-order adds, no bucket counting sort).
   extern __shared__ __align__(16) unsigned char smem[];
   const int lane = lane_id();
   constexpr int M = MODE & 7;
@@ -1384,7 +1366,7 @@ __global__ void __launch_bounds__(kWarpRowThreads, wr_ctas_per_sm(PASS, MODE & 7
     mv = mvn;
     fetch((int64_t)enn, rown, mvn);
     int c = -1;
-    if (M != 1 && (PASS == 1 || M == 3) && !(MODE & 24)) {
+    if (M != 1 && (PASS == 1 || M == 3) && !(MODE & 8)) {
       // rows whose products are (almost) all distinct columns: counting sort on column buckets
       // (esc_kernels.cuh); -1 = uneven buckets, the hash map below takes the row
       const int64_t np = PASS == 0 ? need : __shfl_sync(0xffffffffu, mv_prev6, 6);
