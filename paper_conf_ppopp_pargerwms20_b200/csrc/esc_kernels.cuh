@@ -25,6 +25,8 @@
 // — ~4 instructions per product instead of the 5-step shuffle binary search of expand_row.
 #pragma once
 
+#include <type_traits>
+
 #include "speck_internal.cuh"
 
 namespace speck {
@@ -33,6 +35,16 @@ namespace speck {
 #define SPECK_ESC_LAMBDA 2
 #endif
 constexpr int kEscLambda = SPECK_ESC_LAMBDA;   // target products per bucket
+#ifndef SPECK_ESC_RATIO_PCT
+#define SPECK_ESC_RATIO_PCT 200
+#endif
+// numeric rows take the counting sort when products <= this % of their entries (repeated
+// columns cost the rank passes a second round)
+constexpr int kEscRatioPct = SPECK_ESC_RATIO_PCT;
+#ifndef SPECK_ESC_STAGED
+#define SPECK_ESC_STAGED 1
+#endif
+constexpr bool kEscStaged = SPECK_ESC_STAGED != 0;   // numeric rows: one expansion (esc_row_staged)
 // a row whose largest bucket exceeds this goes back to the hash map: clustered columns (stencil
 // rows: many products on few columns) would make the in-bucket ranking quadratic
 constexpr int kEscMaxBucket = 8 * kEscLambda + 16;
@@ -82,6 +94,7 @@ __device__ __forceinline__ void expand_esc(const SpgemmArgs<V>& p, int64_t a0, i
                                            const PreBatch<V>* pre = nullptr) {
   const int lane = lane_id();
   int rot = 0;
+  int pbase = 0;   // products of the earlier batches (the row's product index of q0 = pbase + q0)
   for (int b0 = 0; b0 < alen; b0 += 32) {
     const int fi = b0 + lane;
     int64_t bst = 0;
@@ -116,6 +129,8 @@ __device__ __forceinline__ void expand_esc(const SpgemmArgs<V>& p, int64_t a0, i
     const int excl = incl - blen;
     const int Pb = __shfl_sync(0xffffffffu, incl, 31);
     const int64_t boff = bst - excl;          // product pp of owner o is B entry boff_o + pp
+    const int pb0 = pbase;
+    pbase += Pb;
     const bool own_any = blen > 0;
     const int nch = (Pb + 31) >> 5;
     int c = (wi - rot) & (nw - 1);
@@ -148,7 +163,10 @@ __device__ __forceinline__ void expand_esc(const SpgemmArgs<V>& p, int64_t a0, i
 #pragma unroll
       for (int u = 0; u < U; ++u) {
         if ((c + u * nw) * 32 >= Pb) continue;                   // warp-uniform
-        f(col[u], av[u] * bv[u], act[u]);
+        if constexpr (std::is_invocable_v<F, uint32_t, V, bool, int>)
+          f(col[u], av[u] * bv[u], act[u], pb0 + (c + u * nw) * 32 + lane);
+        else
+          f(col[u], av[u] * bv[u], act[u]);
       }
     }
   }
@@ -214,7 +232,11 @@ __device__ __forceinline__ int esc_row(const SpgemmArgs<V>& p, unsigned char* re
   const uint32_t lo = (uint32_t)cmin;
   const uint32_t range = (uint32_t)(cmax - cmin + 1);
   const uint64_t mult = range ? ((uint64_t)NB << 32) / range : 0;   // floor: bucket <= (range-1) NB / range < NB
-  auto home = [&](uint32_t col) { return (uint32_t)(((uint64_t)(col - lo) * mult) >> 32); };
+  const uint32_t mlo = (uint32_t)mult, mhi = (uint32_t)(mult >> 32);
+  auto home = [&](uint32_t col) {
+    const uint32_t x = col - lo;
+    return __umulhi(x, mlo) + x * mhi;
+  };
 
   for (int b = t; b < NB; b += T) bc[b] = 0;
   esc_sync<NW>();
@@ -267,7 +289,7 @@ __device__ __forceinline__ int esc_row(const SpgemmArgs<V>& p, unsigned char* re
       const int e = e0 + lane;
       const bool act = e < n;
       const uint32_t k = act ? keys[e] : 0u;
-      const uint32_t b = home(k);
+      const uint32_t b = act ? home(k) : 0u;
       const int s = act ? (b ? bc[b - 1] : 0) : 0, en = act ? bc[b] : 0;
       const int r = esc_rank(keys, s, en, k);
       if (act) {
@@ -317,6 +339,212 @@ __device__ __forceinline__ int esc_row(const SpgemmArgs<V>& p, unsigned char* re
     if (act) {
       const int64_t o = cbase + dc[b] + r;
       p.C_col[o] = (int32_t)kk;
+      p.C_val[o] = vals[e];
+    }
+  }
+  esc_sync<NW>();
+  return cnt;
+}
+
+// ---------------------------------------------------------------------------------------------
+// Numeric rows with ONE expansion ("staged"): the products are gathered once, in product order,
+// into shared memory (column, a*b, arrival index inside the column bucket), the bucket counts are
+// scanned, and a shared-memory-only pass files every product's index under its bucket slot.  The
+// rank/write-out then reads the bucket members through that index.  esc_row's S pass re-expands
+// the row from global memory (A -> B row bounds -> B columns and values again: ~35% of the
+// numeric ESC instructions and a second dependent load chain, ncu profiles/r02/r02u_*); here the
+// second pass touches shared memory only.  Shared memory per product: 4 (column) + sizeof(V) +
+// 2 (slot -> product) + 1 (arrival index) + 8/lambda (bucket starts, distinct starts).
+// ---------------------------------------------------------------------------------------------
+template <typename V>
+__host__ __device__ inline int64_t esc_staged_capacity(int pass, int64_t bytes) {
+  const int64_t per = pass == 0 ? 7 : 7 + (int64_t)sizeof(V);   // bytes per product besides the buckets
+  const int64_t c = (bytes - 320) * kEscLambda / (per * kEscLambda + 8);
+  return c < 65535 ? c : 65535;     // slot -> product indices are 16-bit
+}
+
+// rank of k among keys[idx[s .. en)] (keys < k); warp-uniform trip count as esc_rank
+__device__ __forceinline__ int esc_rank_ind(const uint32_t* keys, const uint16_t* idx, int s, int en, uint32_t k) {
+  const int len = en - s;
+  const int mx = (int)__reduce_max_sync(0xffffffffu, (unsigned)len);
+  int r = 0;
+  for (int d = 0; d < mx; d += 4) {
+#pragma unroll
+    for (int u = 0; u < 4; ++u)
+      if (d + u < len) r += keys[idx[s + d + u]] < k;
+  }
+  return r;
+}
+
+// One row by NW warps (warp wi) in `region`; n = products (<= esc_staged_capacity of the region).
+//   PASS 0: returns the number of distinct columns (every thread).
+//   PASS 1: cnt = exact entries; writes the row sorted at C[cbase, cbase + cnt) and returns cnt.
+// -1: the buckets are too uneven (the caller then takes the hash map on the same region).
+template <int NW, int PASS, typename V>
+__device__ __forceinline__ int esc_row_staged(const SpgemmArgs<V>& p, unsigned char* region, int wi, int64_t a0,
+                                              int alen, int n, int cnt, int32_t cmin, int32_t cmax, int64_t cbase,
+                                              int* red, const PreBatch<V>* pre = nullptr) {
+  const int lane = lane_id();
+  const int t = wi * 32 + lane;
+  constexpr int T = NW * 32;
+  int NB = (n + kEscLambda - 1) / kEscLambda;
+  NB = (NB + 31) & ~31;
+  auto pad16 = [](size_t b) { return (b + 15) & ~(size_t)15; };
+  int* bc = reinterpret_cast<int*>(region);
+  int* dc = bc + NB;
+  uint32_t* keys = reinterpret_cast<uint32_t*>(region + (size_t)NB * 8);
+  V* vals = reinterpret_cast<V*>(reinterpret_cast<unsigned char*>(keys) + pad16((size_t)n * 4));
+  uint16_t* sidx = reinterpret_cast<uint16_t*>(reinterpret_cast<unsigned char*>(vals) +
+                                               (PASS == 1 ? pad16((size_t)n * sizeof(V)) : 0));
+  uint8_t* jb = reinterpret_cast<uint8_t*>(sidx) + pad16((size_t)n * 2);
+  const uint32_t lo = (uint32_t)cmin;
+  const uint32_t range = (uint32_t)(cmax - cmin + 1);
+  const uint64_t mult = range ? ((uint64_t)NB << 32) / range : 0;
+  // bucket = floor((col - lo) * mult / 2^32), written out as high(x * mult_lo) + x * mult_hi
+  const uint32_t mlo = (uint32_t)mult, mhi = (uint32_t)(mult >> 32);
+  auto home = [&](uint32_t col) {
+    const uint32_t x = col - lo;
+    return __umulhi(x, mlo) + x * mhi;
+  };
+  const bool dups = PASS == 1 && n != cnt;
+
+  for (int b = t; b < NB; b += T) {
+    bc[b] = 0;
+    if (dups) dc[b] = 0;
+  }
+  esc_sync<NW>();
+  // ---- G: gather (column, a*b) in product order; count the buckets --------------------------
+  expand_esc<PASS, V, PASS == 0 ? 4 : 2>(p, a0, alen, wi, NW, [&](uint32_t col, V v, bool act, int pi) {
+    if (act) {
+      const int j = atomicAdd(&bc[home(col)], 1);
+      keys[pi] = col;
+      if (PASS == 1) vals[pi] = v;
+      jb[pi] = (uint8_t)(j < 255 ? j : 255);
+    }
+  }, pre);
+  esc_sync<NW>();
+  const int mx = esc_scan<NW>(bc, NB, wi, red);      // bc[b] = first slot of bucket b
+  if (mx > kEscMaxBucket) {
+    if (t == 0) count_path(p.paths, SPECK_PATH_ESC_FALLBACK);
+    return -1;
+  }
+  if (t == 0) count_path(p.paths, PASS == 0 ? SPECK_PATH_SYM_ESC : dups ? SPECK_PATH_NUM_ESC_DUP : SPECK_PATH_NUM_ESC);
+  // ---- F: file every product under its bucket slot (shared memory only) ----------------------
+  for (int e = t; e < n; e += T) sidx[bc[home(keys[e])] + jb[e]] = (uint16_t)e;
+  esc_sync<NW>();
+  auto bend = [&](uint32_t b) { return b + 1 < (uint32_t)NB ? bc[b + 1] : n; };
+  if (PASS == 0) {
+    // distinct columns = entries without an equal key in an earlier slot of their bucket
+    int d = 0;
+    for (int q0 = wi * 32; q0 < n; q0 += T) {
+      const int q = q0 + lane;
+      const bool act = q < n;
+      const uint32_t k = act ? keys[sidx[q]] : 0u;
+      const uint32_t b = act ? home(k) : 0u;
+      const int s = act ? bc[b] : 0, len = act ? q - s : 0;
+      const int mxl = (int)__reduce_max_sync(0xffffffffu, (unsigned)len);
+      bool first = act;
+      for (int j = 0; j < mxl; ++j)
+        if (j < len) first &= keys[sidx[s + j]] != k;
+      d += first;
+    }
+    d = warp_sum(d);
+    if (NW == 1) return d;
+    if (lane == 0) red[2 * NW] = 0;
+    __syncthreads();
+    if (lane == 0) atomicAdd(&red[2 * NW], d);
+    __syncthreads();
+    const int total = red[2 * NW];
+    __syncthreads();
+    return total;
+  }
+  if (!dups) {
+    // sorted position = bucket start + rank in the bucket; slots in bucket order keep the
+    // warp's stores to C nearly contiguous
+    for (int q0 = wi * 32; q0 < n; q0 += T) {        // warp-uniform: every lane calls esc_rank_ind
+      const int q = q0 + lane;
+      const bool act = q < n;
+      const int e = act ? sidx[q] : 0;
+      const uint32_t k = act ? keys[e] : 0u;
+      const uint32_t b = act ? home(k) : 0u;
+      const int s = act ? bc[b] : 0, en = act ? bend(b) : 0;
+      const int r = esc_rank_ind(keys, sidx, s, en, k);
+      if (act) {
+        p.C_col[cbase + s + r] = (int32_t)k;
+        p.C_val[cbase + s + r] = vals[e];
+      }
+    }
+    esc_sync<NW>();
+    return cnt;
+  }
+  // ---- repeated columns (rare: C5 has ~1 per 1000 products, but most large rows have one) ----
+  // R1: one pass over each entry's bucket gives its rank among ALL keys of the bucket (lt), whether
+  // an equal key sits in an earlier slot (then it is a dropped duplicate), and, for the first
+  // occurrence, the sum of its equals; first occurrences count one distinct entry for their
+  // bucket, and a bucket holding any equal pair is flagged (bit 30 of its start).
+  // R2: distinct starts by a scan; an entry of an unflagged bucket is written at distinct start +
+  // lt, only flagged buckets rank again among their first occurrences.
+  constexpr int kDupF = 0x40000000, kBcMask = 0x3fffffff;
+  auto bend2 = [&](uint32_t b) { return b + 1 < (uint32_t)NB ? (bc[b + 1] & kBcMask) : n; };
+  for (int q0 = wi * 32; q0 < n; q0 += T) {           // warp-uniform trip counts inside
+    const int q = q0 + lane;
+    const bool act = q < n;
+    const int e = act ? sidx[q] : 0;
+    const uint32_t k = act ? keys[e] : 0u;
+    const uint32_t b = act ? home(k) : 0u;
+    const int s = act ? (bc[b] & kBcMask) : 0, len = act ? bend2(b) - s : 0;
+    const int mxl = (int)__reduce_max_sync(0xffffffffu, (unsigned)len);
+    int lt = 0;
+    bool earlier = false, eq = false;
+    V sum = V(0);
+    for (int d = 0; d < mxl; ++d) {
+      if (d < len && s + d != q) {
+        const int f = sidx[s + d];
+        const uint32_t kd = keys[f];
+        lt += kd < k;
+        if (kd == k) {
+          eq = true;
+          if (s + d < q) earlier = true;
+          else sum += vals[f];
+        }
+      }
+    }
+    if (act) {
+      if (!earlier) {
+        if (eq) vals[e] += sum;          // the later equals' values are only read here
+        atomicAdd(&dc[b], 1);
+      }
+      if (eq) atomicOr(&bc[b], kDupF);
+      jb[e] = (uint8_t)(lt | (earlier ? 0x80 : 0));
+    }
+  }
+  esc_sync<NW>();
+  esc_scan<NW>(dc, NB, wi, red);      // dc[b] = first distinct position of bucket b
+  for (int q0 = wi * 32; q0 < n; q0 += T) {
+    const int q = q0 + lane;
+    const int e = q < n ? sidx[q] : 0;
+    const int j = q < n ? jb[e] : 0x80;
+    const bool act = !(j & 0x80);
+    const uint32_t k = act ? keys[e] : 0u;
+    const uint32_t b = act ? home(k) : 0u;
+    const int fl = act ? bc[b] : 0;
+    int r = j & 0x7f;
+    const bool flagged = act && (fl & kDupF);
+    if (__any_sync(0xffffffffu, flagged)) {
+      const int s = flagged ? (fl & kBcMask) : 0, len = flagged ? bend2(b) - s : 0;
+      const int mxl = (int)__reduce_max_sync(0xffffffffu, (unsigned)len);
+      int r2 = 0;
+      for (int d = 0; d < mxl; ++d) {
+        if (d < len) {
+          const int f = sidx[s + d];
+          r2 += keys[f] < k && !(jb[f] & 0x80);
+        }
+      }
+      if (flagged) r = r2;
+    }
+    if (act) {
+      const int64_t o = cbase + dc[b] + r;
+      p.C_col[o] = (int32_t)k;
       p.C_val[o] = vals[e];
     }
   }

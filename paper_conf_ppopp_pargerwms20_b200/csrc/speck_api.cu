@@ -888,7 +888,6 @@ speck_status_t spgemm_rows_impl(speck_handle_t h, const speck_csr_t* A, const sp
                                 int64_t r0, int64_t r1, int32_t* C_col, V* C_val, cudaStream_t s) {
   const int64_t m = A->rows;
   if (r1 <= r0 || h->nnz_c == 0) return SPECK_OK;
-  speck_status_t st;
   const int64_t tiles = (m + kBinTile - 1) / kBinTile;
   const BinParams bpn = make_bin_params(h, 1);
   h->st.lb_numeric = 1;

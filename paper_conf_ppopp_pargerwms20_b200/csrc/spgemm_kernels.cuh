@@ -85,7 +85,11 @@ __device__ __forceinline__ uint64_t bkt_mult(uint32_t range, uint32_t S) {
   return range ? (nh << 32) / range : 0;
 }
 __device__ __forceinline__ uint32_t bkt_home(uint32_t col, uint32_t lo, uint64_t mult) {
-  return (uint32_t)(((uint64_t)(col - lo) * mult) >> 32);
+  // floor((col - lo) * mult / 2^32) as high(x * mult_lo) + x * mult_hi: nvcc 12.9 folded the
+  // 64-bit product-and-shift form wrongly inside one loop of esc_row_staged (illegal shared
+  // addresses on every run; the explicit form compiles to IMAD.HI + IMAD)
+  const uint32_t x = col - lo;
+  return __umulhi(x, (uint32_t)mult) + x * (uint32_t)(mult >> 32);
 }
 
 // Insert into the bucketed ordered map (keys 16-byte aligned, NB = S/8 buckets): two 16-byte
@@ -1005,11 +1009,10 @@ __device__ __forceinline__ void spgemm_group(const SpgemmArgs<V>& p, const int64
         // single-row hash blocks whose products are (almost) all distinct: bucket counting sort
         const int64_t ecap = esc_capacity<V>(PASS, kCfgMapBytes[CFG]);
         bm.esc = (nr == 1 && !dense && tot_p > 0 && tot_p <= ecap && tot_p <= 32 * T &&
-                  p.esc >= (PASS == 0 ? 2 : 1) && (PASS == 0 || tot_p <= 2 * tot_c)) ? 1 : 0;
+                  p.esc >= (PASS == 0 ? 2 : 1) && (PASS == 0 || tot_p * 100 <= (int64_t)kEscRatioPct * tot_c)) ? 1 : 0;
       }
     }
     __syncthreads();
-    const int64_t nnzA = bm.nnzA;
     constexpr int NW = T / 32;
 
     int esc_done = 0;
@@ -1020,10 +1023,14 @@ __device__ __forceinline__ void spgemm_group(const SpgemmArgs<V>& p, const int64
         for (int i = tid; i < p.nchunks; i += T) chist[i] = 0;
         __syncthreads();
       }
-      const int c = esc_row<NW, PASS, V>(p, smem, kCfgMapBytes[CFG], warp_id(), bm.astart[0], (int)bm.nnzA,
-                                         (int)bm.prods, (int)bm.cnt, bm.colmin, bm.colmax, bm.cbase[0],
-                                         reinterpret_cast<int*>(bm.scan_part), chunks ? chist : nullptr,
-                                         p.chunk_shift);
+      const int c =
+          (kEscStaged && !chunks && bm.prods <= esc_staged_capacity<V>(PASS, kCfgMapBytes[CFG]))
+              ? esc_row_staged<NW, PASS, V>(p, smem, warp_id(), bm.astart[0], (int)bm.nnzA, (int)bm.prods, (int)bm.cnt,
+                                      bm.colmin, bm.colmax, bm.cbase[0], reinterpret_cast<int*>(bm.scan_part))
+              : esc_row<NW, PASS, V>(p, smem, kCfgMapBytes[CFG], warp_id(), bm.astart[0], (int)bm.nnzA,
+                                     (int)bm.prods, (int)bm.cnt, bm.colmin, bm.colmax, bm.cbase[0],
+                                     reinterpret_cast<int*>(bm.scan_part), chunks ? chist : nullptr,
+                                     p.chunk_shift);
       if (c >= 0) {
         esc_done = 1;
         if (PASS == 0 && tid == 0) p.cnt[bm.row[b0]] = c;
@@ -1370,8 +1377,10 @@ __global__ void __launch_bounds__(kWarpRowThreads, wr_ctas_per_sm(PASS, MODE & 7
       // rows whose products are (almost) all distinct columns: counting sort on column buckets
       // (esc_kernels.cuh); -1 = uneven buckets, the hash map below takes the row
       const int64_t np = PASS == 0 ? need : __shfl_sync(0xffffffffu, mv_prev6, 6);
-      if (p.esc >= (PASS == 0 ? 2 : 1) && np > 0 && np <= esc_cap && (PASS == 0 || np <= 2 * need))
-        c = esc_row<1, PASS, V>(p, region, kRegion, 0, a0, alen, (int)np, (int)need, cmn, cmx, m2, nullptr, nullptr, 0);
+      if (p.esc >= (PASS == 0 ? 2 : 1) && np > 0 && np <= esc_cap && (PASS == 0 || np * 100 <= (int64_t)kEscRatioPct * need))
+        c = (kEscStaged && np <= esc_staged_capacity<V>(PASS, kRegion))
+                ? esc_row_staged<1, PASS, V>(p, region, 0, a0, alen, (int)np, (int)need, cmn, cmx, m2, nullptr, &bcur)
+                : esc_row<1, PASS, V>(p, region, kRegion, 0, a0, alen, (int)np, (int)need, cmn, cmx, m2, nullptr, nullptr, 0);
     }
     if (c < 0)
       c = warp_row<PASS, V, MODE>(p, rk, rv, S, a0, alen, cmn, cmx, (int32_t)(m3 - m2), m2, &bcur,
