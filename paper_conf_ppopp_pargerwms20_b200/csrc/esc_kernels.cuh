@@ -41,6 +41,13 @@ constexpr int kEscLambda = SPECK_ESC_LAMBDA;   // target products per bucket
 // numeric rows take the counting sort when products <= this % of their entries (repeated
 // columns cost the rank passes a second round)
 constexpr int kEscRatioPct = SPECK_ESC_RATIO_PCT;
+#ifndef SPECK_ESC_MAX_CFG
+#define SPECK_ESC_MAX_CFG 4   // block configurations that may take the counting sort (experiments)
+#endif
+#ifndef SPECK_ESC_TABLE
+#define SPECK_ESC_TABLE 1
+#endif
+constexpr bool kEscTable = SPECK_ESC_TABLE != 0;   // block rows: reference table in shared memory
 #ifndef SPECK_ESC_STAGED
 #define SPECK_ESC_STAGED 1
 #endif
@@ -89,86 +96,162 @@ struct PreBatch {
   bool valid = false;
 };
 
+// The chunks of one batch whose references are compacted to lanes [0, nn) (lane o: its
+// products [excl_o, excl_o + len) start at B entry boff_o + excl_o; own_any = len > 0): chunk c of
+// 32 products goes to warp (c + rot) mod nw; the owner of product pp of a chunk is found from one
+// warp-wide OR of the row starts falling into the chunk and a popcount.
+template <int PASS, typename V, int U, typename F>
+__device__ __forceinline__ void esc_batch_chunks(const SpgemmArgs<V>& p, int excl, bool own_any, int64_t boff, V a,
+                                                 int Pb, int pb0, int wi, int nw, int& rot, F& f) {
+  const int lane = lane_id();
+  const int nch = (Pb + 31) >> 5;
+  int c = (wi - rot) & (nw - 1);
+  rot = (rot + nch) & (nw - 1);
+  for (; c < nch; c += U * nw) {
+    uint32_t col[U];
+    V bv[U], av[U];
+    bool act[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const int q0 = (c + u * nw) * 32;
+      col[u] = 0x80000000u | (uint32_t)lane;
+      bv[u] = V(0);
+      av[u] = V(0);
+      act[u] = false;
+      if (q0 >= Pb) continue;                                   // warp-uniform
+      const uint32_t d = (uint32_t)(excl - q0);
+      const uint32_t bits = __reduce_or_sync(0xffffffffu, (own_any && d < 32u) ? (1u << d) : 0u);
+      const int base = __popc(__ballot_sync(0xffffffffu, own_any && excl < q0));
+      const int own = base + __popc(bits & (0xffffffffu >> (31 - lane))) - 1;
+      const int pp = q0 + lane;
+      const int64_t idx = __shfl_sync(0xffffffffu, boff, own) + pp;
+      if (PASS == 1) av[u] = __shfl_sync(0xffffffffu, a, own);
+      act[u] = pp < Pb;
+      if (act[u]) {
+        col[u] = (uint32_t)p.B_col[idx];
+        if (PASS == 1) bv[u] = __ldg(p.B_val + idx);
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      if ((c + u * nw) * 32 >= Pb) continue;                   // warp-uniform
+      if constexpr (std::is_invocable_v<F, uint32_t, V, bool, int>)
+        f(col[u], av[u] * bv[u], act[u], pb0 + (c + u * nw) * 32 + lane);
+      else
+        f(col[u], av[u] * bv[u], act[u]);
+    }
+  }
+}
+
+// One batch of 32 NZ of A_i (NZ [a0 + b0, a0 + b0 + 32) of the row's alen): lane f loads its
+// reference (B row start, length, a), the non-empty references are compacted to the low lanes
+// and scanned.  Returns Pb (products of the batch); excl/boff/a/own_any as esc_batch_chunks wants.
+template <int PASS, typename V>
+__device__ __forceinline__ int esc_batch_setup(const SpgemmArgs<V>& p, int64_t a0, int alen, int b0,
+                                               const PreBatch<V>* pre, int& excl, bool& own_any, int64_t& boff,
+                                               V& a) {
+  const int lane = lane_id();
+  const int fi = b0 + lane;
+  int64_t bst = 0;
+  int blen = 0;
+  a = V(0);
+  if (pre && b0 == 0 && pre->valid) {
+    bst = pre->bst;
+    blen = pre->blen;
+    a = pre->a;
+  } else if (fi < alen) {
+    const int32_t kc = p.A_col[a0 + fi];
+    if (PASS == 1) a = __ldg(p.A_val + a0 + fi);
+    bst = p.B_rp[kc];
+    blen = (int)(p.B_rp[kc + 1] - bst);
+  }
+  const uint32_t ne = __ballot_sync(0xffffffffu, blen > 0);
+  if (!ne) {
+    excl = 0;
+    own_any = false;
+    boff = 0;
+    return 0;
+  }
+  const int nn = __popc(ne);
+  if (ne != (0xffffffffu >> (32 - nn))) {
+    // compact the non-empty references to lanes [0, nn): lane j takes the (j+1)-th set bit
+    int src = 0;
+#pragma unroll
+    for (int step = 16; step > 0; step >>= 1)
+      if (__popc(ne & ((2u << (src + step - 1)) - 1u)) <= lane) src += step;
+    src = min(src, 31);
+    bst = __shfl_sync(0xffffffffu, bst, src);
+    blen = __shfl_sync(0xffffffffu, blen, src);
+    if (PASS == 1) a = __shfl_sync(0xffffffffu, a, src);
+    if (lane >= nn) blen = 0;
+  }
+  const int incl = warp_incl_scan(blen);
+  excl = incl - blen;
+  own_any = blen > 0;
+  boff = bst - excl;          // product pp of owner o is B entry boff_o + pp
+  return __shfl_sync(0xffffffffu, incl, 31);
+}
+
+// Products of A_i (NZ [a0, a0 + alen)) for warp wi of nw (a power of two): every warp sets up
+// every batch of 32 NZ, chunks of 32 products rotate over the warps across batches.
+// f(col, a*b, active[, product index]) is called by all 32 lanes.  `pre` (optional): the row's
+// first batch, loaded ahead by the caller (lane f: B row start / length and a of the row's f-th NZ).
 template <int PASS, typename V, int U, typename F>
 __device__ __forceinline__ void expand_esc(const SpgemmArgs<V>& p, int64_t a0, int alen, int wi, int nw, F&& f,
                                            const PreBatch<V>* pre = nullptr) {
-  const int lane = lane_id();
   int rot = 0;
   int pbase = 0;   // products of the earlier batches (the row's product index of q0 = pbase + q0)
   for (int b0 = 0; b0 < alen; b0 += 32) {
-    const int fi = b0 + lane;
-    int64_t bst = 0;
-    int blen = 0;
-    V a = V(0);
-    if (pre && b0 == 0 && pre->valid) {
-      bst = pre->bst;
-      blen = pre->blen;
-      a = pre->a;
-    } else if (fi < alen) {
-      const int32_t kc = p.A_col[a0 + fi];
-      if (PASS == 1) a = __ldg(p.A_val + a0 + fi);
-      bst = p.B_rp[kc];
-      blen = (int)(p.B_rp[kc + 1] - bst);
-    }
-    const uint32_t ne = __ballot_sync(0xffffffffu, blen > 0);
-    if (!ne) continue;
-    const int nn = __popc(ne);
-    if (ne != (0xffffffffu >> (32 - nn))) {
-      // compact the non-empty references to lanes [0, nn): lane j takes the (j+1)-th set bit
-      int src = 0;
-#pragma unroll
-      for (int step = 16; step > 0; step >>= 1)
-        if (__popc(ne & ((2u << (src + step - 1)) - 1u)) <= lane) src += step;
-      src = min(src, 31);
-      bst = __shfl_sync(0xffffffffu, bst, src);
-      blen = __shfl_sync(0xffffffffu, blen, src);
-      if (PASS == 1) a = __shfl_sync(0xffffffffu, a, src);
-      if (lane >= nn) blen = 0;
-    }
-    const int incl = warp_incl_scan(blen);
-    const int excl = incl - blen;
-    const int Pb = __shfl_sync(0xffffffffu, incl, 31);
-    const int64_t boff = bst - excl;          // product pp of owner o is B entry boff_o + pp
-    const int pb0 = pbase;
+    int excl;
+    bool own_any;
+    int64_t boff;
+    V a;
+    const int Pb = esc_batch_setup<PASS, V>(p, a0, alen, b0, pre, excl, own_any, boff, a);
+    if (!Pb) continue;
+    esc_batch_chunks<PASS, V, U>(p, excl, own_any, boff, a, Pb, pbase, wi, nw, rot, f);
     pbase += Pb;
-    const bool own_any = blen > 0;
-    const int nch = (Pb + 31) >> 5;
-    int c = (wi - rot) & (nw - 1);
-    rot = (rot + nch) & (nw - 1);
-    for (; c < nch; c += U * nw) {
-      uint32_t col[U];
-      V bv[U], av[U];
-      bool act[U];
-#pragma unroll
-      for (int u = 0; u < U; ++u) {
-        const int q0 = (c + u * nw) * 32;
-        col[u] = 0x80000000u | (uint32_t)lane;
-        bv[u] = V(0);
-        av[u] = V(0);
-        act[u] = false;
-        if (q0 >= Pb) continue;                                   // warp-uniform
-        const uint32_t d = (uint32_t)(excl - q0);
-        const uint32_t bits = __reduce_or_sync(0xffffffffu, (own_any && d < 32u) ? (1u << d) : 0u);
-        const int base = __popc(__ballot_sync(0xffffffffu, own_any && excl < q0));
-        const int own = base + __popc(bits & (0xffffffffu >> (31 - lane))) - 1;
-        const int pp = q0 + lane;
-        const int64_t idx = __shfl_sync(0xffffffffu, boff, own) + pp;
-        if (PASS == 1) av[u] = __shfl_sync(0xffffffffu, a, own);
-        act[u] = pp < Pb;
-        if (act[u]) {
-          col[u] = (uint32_t)p.B_col[idx];
-          if (PASS == 1) bv[u] = __ldg(p.B_val + idx);
-        }
-      }
-#pragma unroll
-      for (int u = 0; u < U; ++u) {
-        if ((c + u * nw) * 32 >= Pb) continue;                   // warp-uniform
-        if constexpr (std::is_invocable_v<F, uint32_t, V, bool, int>)
-          f(col[u], av[u] * bv[u], act[u], pb0 + (c + u * nw) * 32 + lane);
-        else
-          f(col[u], av[u] * bv[u], act[u]);
-      }
-    }
+  }
+}
+
+// Shared-memory reference table of a row (block rows): bytes for nb = ceil(alen / 32) batches.
+template <typename V>
+__host__ __device__ inline int64_t esc_tbl_bytes(int alen) {
+  const int64_t nb = (alen + 31) / 32;
+  return nb * 32 * (8 + 4 + (int64_t)sizeof(V)) + ((nb * 4 + 15) & ~(int64_t)15);
+}
+// As expand_esc for the NW warps of a block, but every batch is set up once: warp w sets up
+// batches w, w + NW, ... into the table `tbl` (esc_tbl_bytes, 16-byte aligned) in parallel, then
+// all warps stream the chunks from it (one dependent A -> B-row-bounds round trip per row instead
+// of one per batch per warp).  Barrier inside.
+template <int PASS, typename V, int NW, int U, typename F>
+__device__ __forceinline__ void expand_tbl(const SpgemmArgs<V>& p, int64_t a0, int alen, int wi, unsigned char* tbl,
+                                           F&& f) {
+  const int lane = lane_id();
+  const int nb = (alen + 31) >> 5;
+  int64_t* tboff = reinterpret_cast<int64_t*>(tbl);
+  int* texcl = reinterpret_cast<int*>(tboff + nb * 32);
+  V* ta = reinterpret_cast<V*>(texcl + nb * 32);
+  int* tpb = reinterpret_cast<int*>(ta + nb * 32);
+  for (int j = wi; j < nb; j += NW) {
+    int excl;
+    bool own_any;
+    int64_t boff;
+    V a;
+    const int Pb = esc_batch_setup<PASS, V>(p, a0, alen, j * 32, nullptr, excl, own_any, boff, a);
+    tboff[j * 32 + lane] = boff;
+    texcl[j * 32 + lane] = own_any ? excl : 0x7fffffff;
+    if (PASS == 1) ta[j * 32 + lane] = a;
+    if (lane == 0) tpb[j] = Pb;
+  }
+  __syncthreads();
+  int rot = 0, pbase = 0;
+  for (int j = 0; j < nb; ++j) {
+    const int Pb = tpb[j];
+    if (!Pb) continue;
+    const int ex = texcl[j * 32 + lane];
+    const V a = PASS == 1 ? ta[j * 32 + lane] : V(0);
+    esc_batch_chunks<PASS, V, U>(p, ex, ex != 0x7fffffff, tboff[j * 32 + lane], a, Pb, pbase, wi, NW, rot, f);
+    pbase += Pb;
   }
 }
 
@@ -381,9 +464,9 @@ __device__ __forceinline__ int esc_rank_ind(const uint32_t* keys, const uint16_t
 //   PASS 1: cnt = exact entries; writes the row sorted at C[cbase, cbase + cnt) and returns cnt.
 // -1: the buckets are too uneven (the caller then takes the hash map on the same region).
 template <int NW, int PASS, typename V>
-__device__ __forceinline__ int esc_row_staged(const SpgemmArgs<V>& p, unsigned char* region, int wi, int64_t a0,
-                                              int alen, int n, int cnt, int32_t cmin, int32_t cmax, int64_t cbase,
-                                              int* red, const PreBatch<V>* pre = nullptr) {
+__device__ __forceinline__ int esc_row_staged(const SpgemmArgs<V>& p, unsigned char* region, uint32_t region_bytes,
+                                              int wi, int64_t a0, int alen, int n, int cnt, int32_t cmin,
+                                              int32_t cmax, int64_t cbase, int* red, const PreBatch<V>* pre = nullptr) {
   const int lane = lane_id();
   const int t = wi * 32 + lane;
   constexpr int T = NW * 32;
@@ -414,14 +497,19 @@ __device__ __forceinline__ int esc_row_staged(const SpgemmArgs<V>& p, unsigned c
   }
   esc_sync<NW>();
   // ---- G: gather (column, a*b) in product order; count the buckets --------------------------
-  expand_esc<PASS, V, PASS == 0 ? 4 : 2>(p, a0, alen, wi, NW, [&](uint32_t col, V v, bool act, int pi) {
+  auto gather = [&](uint32_t col, V v, bool act, int pi) {
     if (act) {
       const int j = atomicAdd(&bc[home(col)], 1);
       keys[pi] = col;
       if (PASS == 1) vals[pi] = v;
       jb[pi] = (uint8_t)(j < 255 ? j : 255);
     }
-  }, pre);
+  };
+  unsigned char* tbl = jb + pad16((size_t)n);
+  if (NW > 1 && kEscTable && (size_t)(tbl - region) + (size_t)esc_tbl_bytes<V>(alen) <= region_bytes)
+    expand_tbl<PASS, V, NW, PASS == 0 ? 4 : 2>(p, a0, alen, wi, tbl, gather);   // batches set up once per row
+  else
+    expand_esc<PASS, V, PASS == 0 ? 4 : 2>(p, a0, alen, wi, NW, gather, pre);
   esc_sync<NW>();
   const int mx = esc_scan<NW>(bc, NB, wi, red);      // bc[b] = first slot of bucket b
   if (mx > kEscMaxBucket) {

@@ -1008,7 +1008,7 @@ __device__ __forceinline__ void spgemm_group(const SpgemmArgs<V>& p, const int64
         bm.dense = dense;
         // single-row hash blocks whose products are (almost) all distinct: bucket counting sort
         const int64_t ecap = esc_capacity<V>(PASS, kCfgMapBytes[CFG]);
-        bm.esc = (nr == 1 && !dense && tot_p > 0 && tot_p <= ecap && tot_p <= 32 * T &&
+        bm.esc = (nr == 1 && !dense && tot_p > 0 && tot_p <= ecap && tot_p <= 32 * T && CFG <= SPECK_ESC_MAX_CFG &&
                   p.esc >= (PASS == 0 ? 2 : 1) && (PASS == 0 || tot_p * 100 <= (int64_t)kEscRatioPct * tot_c)) ? 1 : 0;
       }
     }
@@ -1025,7 +1025,7 @@ __device__ __forceinline__ void spgemm_group(const SpgemmArgs<V>& p, const int64
       }
       const int c =
           (kEscStaged && !chunks && bm.prods <= esc_staged_capacity<V>(PASS, kCfgMapBytes[CFG]))
-              ? esc_row_staged<NW, PASS, V>(p, smem, warp_id(), bm.astart[0], (int)bm.nnzA, (int)bm.prods, (int)bm.cnt,
+              ? esc_row_staged<NW, PASS, V>(p, smem, kCfgMapBytes[CFG], warp_id(), bm.astart[0], (int)bm.nnzA, (int)bm.prods, (int)bm.cnt,
                                       bm.colmin, bm.colmax, bm.cbase[0], reinterpret_cast<int*>(bm.scan_part))
               : esc_row<NW, PASS, V>(p, smem, kCfgMapBytes[CFG], warp_id(), bm.astart[0], (int)bm.nnzA,
                                      (int)bm.prods, (int)bm.cnt, bm.colmin, bm.colmax, bm.cbase[0],
@@ -1379,7 +1379,7 @@ __global__ void __launch_bounds__(kWarpRowThreads, wr_ctas_per_sm(PASS, MODE & 7
       const int64_t np = PASS == 0 ? need : __shfl_sync(0xffffffffu, mv_prev6, 6);
       if (p.esc >= (PASS == 0 ? 2 : 1) && np > 0 && np <= esc_cap && (PASS == 0 || np * 100 <= (int64_t)kEscRatioPct * need))
         c = (kEscStaged && np <= esc_staged_capacity<V>(PASS, kRegion))
-                ? esc_row_staged<1, PASS, V>(p, region, 0, a0, alen, (int)np, (int)need, cmn, cmx, m2, nullptr, &bcur)
+                ? esc_row_staged<1, PASS, V>(p, region, kRegion, 0, a0, alen, (int)np, (int)need, cmn, cmx, m2, nullptr, &bcur)
                 : esc_row<1, PASS, V>(p, region, kRegion, 0, a0, alen, (int)np, (int)need, cmn, cmx, m2, nullptr, nullptr, 0);
     }
     if (c < 0)
