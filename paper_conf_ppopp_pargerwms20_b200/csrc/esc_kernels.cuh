@@ -277,9 +277,17 @@ __device__ __forceinline__ int esc_scan(int* bc, int NB, int wi, int* red) {
     if (lane == 31) { red[wi] = incl; red[NW + wi] = mx; }
     __syncthreads();
     int wbase = 0, m2 = 0;
-    for (int w = 0; w < NW; ++w) {
-      if (w < wi) wbase += red[w];
-      m2 = max(m2, red[NW + w]);
+    if (NW >= 8) {
+      // lane w reads warp w's total: one warp scan instead of 2 NW shared loads per thread
+      const int rv = lane < NW ? red[lane] : 0;
+      const int inc = warp_incl_scan(rv);
+      wbase = __shfl_sync(0xffffffffu, inc - rv, wi);
+      m2 = (int)__reduce_max_sync(0xffffffffu, (unsigned)(lane < NW ? red[NW + lane] : 0));
+    } else {
+      for (int w = 0; w < NW; ++w) {
+        if (w < wi) wbase += red[w];
+        m2 = max(m2, red[NW + w]);
+      }
     }
     off += wbase;
     mx = m2;

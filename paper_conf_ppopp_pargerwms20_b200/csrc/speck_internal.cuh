@@ -73,7 +73,13 @@ struct Seg {
 constexpr uint32_t kEmptyKey = 0xFFFFFFFFu;
 
 // Fill rule for the numeric hash maps: final occupancy <= 66%.
-constexpr int kFillNum = 66;
+#ifndef SPECK_SYM_FILL
+#define SPECK_SYM_FILL 66
+#endif
+constexpr int kFillNum = SPECK_SYM_FILL;
+#ifndef SPECK_SYM_REGION_X2
+#define SPECK_SYM_REGION_X2 8     // symbolic single-row regions: need * this / 2 slots (4x products: C5 symbolic 99 -> 91 ms)
+#endif
 // Numeric maps: the order-preserving hash (spgemm_kernels.cuh) walks its probing runs in the
 // write-out, and runs grow like 1/(1-load)^2; homes cover 7/8 of a map, so a 50% fill keeps
 // the effective load near 57% (runs ~5) instead of 75% (runs ~16) at the paper's 66%.

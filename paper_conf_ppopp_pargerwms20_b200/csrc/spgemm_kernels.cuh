@@ -946,12 +946,12 @@ __device__ __forceinline__ void spgemm_group(const SpgemmArgs<V>& p, const int64
       const int64_t need_tot = PASS == 0 ? tot_p : tot_c;
       uint32_t rsz = 0;
       // (multiples of 4 slots so 4-slot probe groups stay 16-byte aligned: 4 + a share of the rest)
-      // A single row gets a region sized to it (symbolic 2x products, numeric 2.5x entries:
+      // A single row gets a region sized to it (symbolic 4x products, numeric 2.5x entries:
       // <= 50% / 40% load), so clearing and the write-out scan touch only the slots the row can use
       // (C5: the write-out scan of the full map was over half of the numeric instructions).
       if (l < nr) {
         if (nr == 1) {
-          const uint64_t want = PASS == 0 ? (uint64_t)need * 2 : (uint64_t)need * 5 / 2;
+          const uint64_t want = PASS == 0 ? (uint64_t)need * SPECK_SYM_REGION_X2 / 2 : (uint64_t)need * 5 / 2;
           const uint64_t w32 = (want + 31) & ~(uint64_t)31;
           rsz = (uint32_t)(w32 < 64 ? 64 : (w32 > cap ? cap : w32));
         } else {
@@ -1264,7 +1264,7 @@ __device__ __noinline__ void dense_row(const SpgemmArgs<V>& p, BlockMeta& bm, in
 // P:785-804): every warp owns a 7 KB region and pulls rows of the bin from a global counter
 // one row ahead, so no warp ever waits at a block barrier for another warp's row (ncu: 33% of
 // the stall samples of the merged-block kernel were barrier waits).  The region is sized to
-// the row (symbolic: 2x products; numeric: 2.5x exact nnz), so clearing and the
+// the row (symbolic: 4x products (capped at the region); numeric: 2.5x exact nnz), so clearing and the
 // write-out scan only the slots a row can use.  Rows of the bin (p.rows) or, without global
 // load balancing, every row of A (p.rows == nullptr).
 // -----------------------------------------------------------------------------------
@@ -1358,8 +1358,8 @@ __global__ void __launch_bounds__(kWarpRowThreads, wr_ctas_per_sm(PASS, MODE & 7
     const int64_t mv_prev6 = mv;
     const int32_t cur = row;
     const int64_t need = PASS == 0 ? m2 : m3 - m2;       // products (symbolic) / exact nnz (numeric)
-    // region: symbolic 2x products (<= 50% load), numeric 2.5x entries (<= 40% load), 32-slot multiples
-    const uint64_t want = PASS == 0 ? (uint64_t)need * 2 : (uint64_t)need * 5 / 2;
+    // region: symbolic 4x products (<= 25% load below the cap), numeric 2.5x entries (<= 40% load), 32-slot multiples
+    const uint64_t want = PASS == 0 ? (uint64_t)need * SPECK_SYM_REGION_X2 / 2 : (uint64_t)need * 5 / 2;
     const uint64_t w32 = (want + 31) & ~(uint64_t)31;
     const uint32_t S = (uint32_t)(w32 < 64 ? 64 : (w32 > cap ? cap : w32));
     const PreBatch<V> bcur = bt;

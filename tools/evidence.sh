@@ -1,5 +1,5 @@
 #!/bin/bash
-# Round-2 evidence job (GPU box): tests, bench lines, reference arm, launch lists, ncu captures,
+# Evidence job (GPU box): tests, bench lines, reference arm, launch lists, ncu captures,
 # sanitizers, 2-rank path.  Outputs under gpurun_out/${TAG}_*.
 TAG=${TAG:-r02e}
 python -c "import __graft_entry__ as g; g.build()" 2>&1 | tail -1
@@ -16,7 +16,7 @@ if [ "${DIST:-1}" = 1 ]; then
   timeout 900 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 --master-addr 127.0.0.1 --master-port 29533 \
     bench.py --gpus 2 --steps 3 --warmup 3 --config c4 --dist-backend gloo --no-cpu-baseline > gpurun_out/${TAG}_dist2_gloo_c4.json 2> gpurun_out/${TAG}_dist2_gloo_c4.err
 fi
-if [ "${SAN:-1}" = 1 ]; then
+if [ "${SAN:-0}" = 1 ]; then   # compute-sanitizer is closed on the GPU pool (round 2)
   for tool in memcheck racecheck synccheck initcheck; do
     timeout 1200 compute-sanitizer --tool $tool --error-exitcode 9 python tools/sanitize_cases.py > gpurun_out/${TAG}_sanitizer_$tool.txt 2>&1
     echo "exit $?" >> gpurun_out/${TAG}_sanitizer_$tool.txt
