@@ -238,11 +238,33 @@ __device__ __forceinline__ uint32_t probe_insert_grp(uint32_t* keys, uint32_t S,
   }
 }
 
-// symbolic insert: true if the key was new
+// symbolic insert: true if the key was new.  Same probe sequence as probe_insert_grp, with the
+// group's matches and empty slots as 4-bit masks (two branches per group instead of eight).
 __device__ __forceinline__ bool hash_insert_key(uint32_t* keys, uint32_t S, uint32_t col) {
+#if SPECK_SYM_PROBE_MASK
+  const uint32_t S4 = S & ~3u;
+  uint32_t g = hash_slot(col, S4) & ~3u;
+  const uint32_t sb = (uint32_t)__cvta_generic_to_shared(keys);
+  while (true) {
+    uint32_t x, y, z, w;
+    asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(x), "=r"(y), "=r"(z), "=r"(w) : "r"(sb + 4u * g));
+    if ((x == col) | (y == col) | (z == col) | (w == col)) return false;
+    const uint32_t em = (x == kEmptyKey ? 1u : 0u) | (y == kEmptyKey ? 2u : 0u) | (z == kEmptyKey ? 4u : 0u) |
+                        (w == kEmptyKey ? 8u : 0u);
+    if (em) {
+      const uint32_t old = atomicCAS(&keys[g + __ffs(em) - 1], kEmptyKey, col);
+      if (old == kEmptyKey) return true;
+      if (old == col) return false;
+      continue;   // another key took the slot: re-read the group
+    }
+    g += 4;
+    if (g >= S4) g = 0;
+  }
+#else
   bool is_new;
   probe_insert_grp(keys, S, col, &is_new);
   return is_new;
+#endif
 }
 
 // Bitonic sort of (keys, vals)[0, n) ascending in shared memory, any n: the "flip"

@@ -316,6 +316,23 @@ def test_row_products_and_allocators(dev):
     h.close()
 
 
+@pytest.mark.parametrize("dt", [torch.float32, torch.float64])
+@pytest.mark.parametrize("amax", [40, 400, 1500])
+def test_counting_sort_rows_block_and_repeats(dev, dt, amax):
+    """Rows of mostly distinct columns in every block configuration (staged counting sort, the
+    shared reference table) with a few repeated columns per row (the flagged-bucket rank pass):
+    B rows of 30-66 entries over 400k columns; A rows of 2-40/400/1500 references."""
+    A = W.uniform_rows(600, 20_000, 2, amax, seed=91, dtype=dt)
+    B = W.uniform_rows(20_000, 400_000, 30, 66, seed=92, dtype=dt)
+    h = sp.Handle(0, path_counters=1)
+    C = h.spgemm(A.to(dev), B.to(dev))
+    torch.cuda.synchronize()
+    paths = h.stats()["paths"]
+    h.close()
+    assert paths["num_esc"] + paths["num_esc_dup"] > 0, paths
+    assert_parity(A, B, C)
+
+
 def test_fig5_dense_window_of_three(dev):
     """Fig. 5: one row, 6 columns, window 3, products at c0,c2,c4,c4,c5 -> c0=1 c2=1 c4=2 c5=1."""
     kv, _ = golden("fig5_dense.txt")

@@ -23,7 +23,7 @@ if [ "${SAN:-0}" = 1 ]; then   # compute-sanitizer is closed on the GPU pool (ro
   done
 fi
 if [ "${NCU:-1}" = 1 ]; then
-  CFG=c5 TAG=${TAG} LAUNCHES=1 K="k_spgemm<.int.1, .int.1, float>;k_spgemm<.int.1, .int.0, float>;k_spgemm<.int.2, .int.1, float>;k_warp_rows<.int.1, float, .int.2>;k_warp_rows<.int.0, float, .int.0>" bash tools/gpu_profile.sh
+  CFG=c5 TAG=${TAG} LAUNCHES=1 K="k_spgemm<.int.1, .int.1, float>;k_spgemm<.int.1, .int.0, float>;k_spgemm<.int.2, .int.1, float>;k_spgemm<.int.3, .int.1, float>;k_spgemm<.int.4, .int.1, float>;k_warp_rows<.int.1, float, .int.2>;k_warp_rows<.int.0, float, .int.0>" bash tools/gpu_profile.sh
   CFG=c3 TAG=${TAG} LAUNCHES=1 K="k_long_bitmap<float>;k_spgemm<.int.4, .int.0, float>" bash tools/gpu_profile.sh
   CFG=c2 TAG=${TAG} LAUNCHES=1 K="k_warp_rows<.int.1, double, .int.1>;k_warp_rows<.int.0, double, .int.0>" bash tools/gpu_profile.sh
 fi

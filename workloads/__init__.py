@@ -302,6 +302,16 @@ def random_sparse(rows: int, cols: int, density: float, seed: int, dtype=torch.f
     return csr_from_coo(rows, cols, r, c, v, dtype=dtype, dedup=False)
 
 
+def uniform_rows(rows: int, cols: int, lmin: int, lmax: int, seed: int, dtype=torch.float32, device="cpu") -> CSR:
+    """Rows of lmin..lmax uniform random columns (row length uniform in [lmin, lmax]; columns drawn
+    with replacement, repeated draws merged, so a row may come out slightly shorter)."""
+    span = lmax - lmin + 1
+    L = lmin + (splitmix64(seed, 1, torch.arange(rows, device=device)) & ((1 << 62) - 1)) % span
+    r = torch.repeat_interleave(torch.arange(rows, device=device), L)
+    c = (splitmix64(seed, 2, torch.arange(r.numel(), device=device)) & ((1 << 62) - 1)) % cols
+    return csr_from_coo(rows, cols, r, c, None, dtype=dtype, seed=seed, stream=3)
+
+
 CONFIGS = {
     "c1": "2D 5-point Poisson 64x64, A*A, fp64",
     "c2": "3D 27-point 128^3 AMG Galerkin R*(A*P), fp64",
