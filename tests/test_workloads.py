@@ -56,3 +56,14 @@ def test_transpose_roundtrip():
     A = W.random_sparse(37, 53, 0.1, seed=2, zero_frac=0.2)
     T = W.transpose(W.transpose(A))
     assert torch.equal(T.row_ptr, A.row_ptr) and torch.equal(T.col, A.col) and torch.equal(T.val, A.val)
+
+
+def test_uniform_rows():
+    A = W.uniform_rows(500, 100_000, 3, 40, seed=5)
+    B = W.uniform_rows(500, 100_000, 3, 40, seed=5)
+    assert torch.equal(A.row_ptr, B.row_ptr) and torch.equal(A.col, B.col) and torch.equal(A.val, B.val)
+    lens = (A.row_ptr[1:] - A.row_ptr[:-1])
+    assert int(lens.min()) >= 1 and int(lens.max()) <= 40 and abs(float(lens.double().mean()) - 21.5) < 2
+    for i in range(0, 500, 50):                    # sorted, distinct, in range
+        c = A.col[A.row_ptr[i]:A.row_ptr[i + 1]]
+        assert bool((c[1:] > c[:-1]).all()) and int(c.min()) >= 0 and int(c.max()) < 100_000
