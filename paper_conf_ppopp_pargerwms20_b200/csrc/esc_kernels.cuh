@@ -503,7 +503,9 @@ __device__ __forceinline__ int esc_row_staged(const SpgemmArgs<V>& p, unsigned c
     bc[b] = 0;
     if (dups) dc[b] = 0;
   }
-  esc_sync<NW>();
+  unsigned char* tbl = jb + pad16((size_t)n);
+  const bool use_tbl = NW > 1 && kEscTable && (size_t)(tbl - region) + (size_t)esc_tbl_bytes<V>(alen) <= region_bytes;
+  if (!use_tbl) esc_sync<NW>();     // (expand_tbl's barrier after the table build orders the clearing)
   // ---- G: gather (column, a*b) in product order; count the buckets --------------------------
   auto gather = [&](uint32_t col, V v, bool act, int pi) {
     if (act) {
@@ -513,8 +515,7 @@ __device__ __forceinline__ int esc_row_staged(const SpgemmArgs<V>& p, unsigned c
       jb[pi] = (uint8_t)(j < 255 ? j : 255);
     }
   };
-  unsigned char* tbl = jb + pad16((size_t)n);
-  if (NW > 1 && kEscTable && (size_t)(tbl - region) + (size_t)esc_tbl_bytes<V>(alen) <= region_bytes)
+  if (use_tbl)
     expand_tbl<PASS, V, NW, PASS == 0 ? 4 : 2>(p, a0, alen, wi, tbl, gather);   // batches set up once per row
   else
     expand_esc<PASS, V, PASS == 0 ? 4 : 2>(p, a0, alen, wi, NW, gather, pre);
@@ -570,7 +571,7 @@ __device__ __forceinline__ int esc_row_staged(const SpgemmArgs<V>& p, unsigned c
         p.C_val[cbase + s + r] = vals[e];
       }
     }
-    esc_sync<NW>();
+    if (NW == 1) esc_sync<NW>();   // block rows: the caller's barrier follows
     return cnt;
   }
   // ---- repeated columns (rare: C5 has ~1 per 1000 products, but most large rows have one) ----
@@ -644,7 +645,7 @@ __device__ __forceinline__ int esc_row_staged(const SpgemmArgs<V>& p, unsigned c
       p.C_val[o] = vals[e];
     }
   }
-  esc_sync<NW>();
+  if (NW == 1) esc_sync<NW>();     // block rows: the caller's barrier follows
   return cnt;
 }
 
