@@ -146,10 +146,20 @@ __device__ __forceinline__ void esc_batch_chunks(const SpgemmArgs<V>& p, int exc
 // One batch of 32 NZ of A_i (NZ [a0 + b0, a0 + b0 + 32) of the row's alen): lane f loads its
 // reference (B row start, length, a), the non-empty references are compacted to the low lanes
 // and scanned.  Returns Pb (products of the batch); excl/boff/a/own_any as esc_batch_chunks wants.
+// first entry >= x of the sorted columns col[l, h)
+__device__ __forceinline__ int64_t esc_lower_bound(const int32_t* __restrict__ col, int64_t l, int64_t h, uint32_t x) {
+  while (l < h) {
+    const int64_t m = (l + h) >> 1;
+    if ((uint32_t)col[m] < x) l = m + 1;
+    else h = m;
+  }
+  return l;
+}
+
 template <int PASS, typename V>
 __device__ __forceinline__ int esc_batch_setup(const SpgemmArgs<V>& p, int64_t a0, int alen, int b0,
                                                const PreBatch<V>* pre, int& excl, bool& own_any, int64_t& boff,
-                                               V& a) {
+                                               V& a, bool clip = false, uint32_t clo = 0, uint32_t chi = 0) {
   const int lane = lane_id();
   const int fi = b0 + lane;
   int64_t bst = 0;
@@ -164,6 +174,13 @@ __device__ __forceinline__ int esc_batch_setup(const SpgemmArgs<V>& p, int64_t a
     if (PASS == 1) a = __ldg(p.A_val + a0 + fi);
     bst = p.B_rp[kc];
     blen = (int)(p.B_rp[kc + 1] - bst);
+    if (clip && blen > 0) {
+      // column segment [clo, chi) of a long row: only the part of B_k inside it
+      const int64_t s0 = esc_lower_bound(p.B_col, bst, bst + blen, clo);
+      const int64_t e0 = esc_lower_bound(p.B_col, s0, bst + blen, chi);
+      bst = s0;
+      blen = (int)(e0 - s0);
+    }
   }
   const uint32_t ne = __ballot_sync(0xffffffffu, blen > 0);
   if (!ne) {
@@ -223,36 +240,62 @@ __host__ __device__ inline int64_t esc_tbl_bytes(int alen) {
 // batches w, w + NW, ... into the table `tbl` (esc_tbl_bytes, 16-byte aligned) in parallel, then
 // all warps stream the chunks from it (one dependent A -> B-row-bounds round trip per row instead
 // of one per batch per warp).  Barrier inside.
-template <int PASS, typename V, int NW, int U, typename F>
-__device__ __forceinline__ void expand_tbl(const SpgemmArgs<V>& p, int64_t a0, int alen, int wi, unsigned char* tbl,
-                                           F&& f) {
+template <typename V>
+struct EscTbl {
+  int64_t* boff;
+  int* excl;
+  V* a;
+  int* pb;
+  __device__ __forceinline__ EscTbl(unsigned char* tbl, int alen) {
+    const int nb = (alen + 31) >> 5;
+    boff = reinterpret_cast<int64_t*>(tbl);
+    excl = reinterpret_cast<int*>(boff + nb * 32);
+    a = reinterpret_cast<V*>(excl + nb * 32);
+    pb = reinterpret_cast<int*>(a + nb * 32);
+  }
+};
+// Reference table of a row: warp w sets up batches w, w + NW, ... (clip: only B entries with
+// columns in [clo, chi)).  Barrier at the end.
+template <int PASS, typename V, int NW>
+__device__ __forceinline__ void esc_tbl_build(const SpgemmArgs<V>& p, int64_t a0, int alen, int wi, unsigned char* tbl,
+                                              bool clip = false, uint32_t clo = 0, uint32_t chi = 0) {
   const int lane = lane_id();
   const int nb = (alen + 31) >> 5;
-  int64_t* tboff = reinterpret_cast<int64_t*>(tbl);
-  int* texcl = reinterpret_cast<int*>(tboff + nb * 32);
-  V* ta = reinterpret_cast<V*>(texcl + nb * 32);
-  int* tpb = reinterpret_cast<int*>(ta + nb * 32);
+  EscTbl<V> t(tbl, alen);
   for (int j = wi; j < nb; j += NW) {
     int excl;
     bool own_any;
     int64_t boff;
     V a;
-    const int Pb = esc_batch_setup<PASS, V>(p, a0, alen, j * 32, nullptr, excl, own_any, boff, a);
-    tboff[j * 32 + lane] = boff;
-    texcl[j * 32 + lane] = own_any ? excl : 0x7fffffff;
-    if (PASS == 1) ta[j * 32 + lane] = a;
-    if (lane == 0) tpb[j] = Pb;
+    const int Pb = esc_batch_setup<PASS, V>(p, a0, alen, j * 32, nullptr, excl, own_any, boff, a, clip, clo, chi);
+    t.boff[j * 32 + lane] = boff;
+    t.excl[j * 32 + lane] = own_any ? excl : 0x7fffffff;
+    if (PASS == 1) t.a[j * 32 + lane] = a;
+    if (lane == 0) t.pb[j] = Pb;
   }
   __syncthreads();
+}
+// Chunks of every batch of a built table, rotated over the NW warps.
+template <int PASS, typename V, int NW, int U, typename F>
+__device__ __forceinline__ void esc_tbl_gather(const SpgemmArgs<V>& p, int alen, int wi, const unsigned char* tbl, F&& f) {
+  const int lane = lane_id();
+  const int nb = (alen + 31) >> 5;
+  EscTbl<V> t(const_cast<unsigned char*>(tbl), alen);
   int rot = 0, pbase = 0;
   for (int j = 0; j < nb; ++j) {
-    const int Pb = tpb[j];
+    const int Pb = t.pb[j];
     if (!Pb) continue;
-    const int ex = texcl[j * 32 + lane];
-    const V a = PASS == 1 ? ta[j * 32 + lane] : V(0);
-    esc_batch_chunks<PASS, V, U>(p, ex, ex != 0x7fffffff, tboff[j * 32 + lane], a, Pb, pbase, wi, NW, rot, f);
+    const int ex = t.excl[j * 32 + lane];
+    const V a = PASS == 1 ? t.a[j * 32 + lane] : V(0);
+    esc_batch_chunks<PASS, V, U>(p, ex, ex != 0x7fffffff, t.boff[j * 32 + lane], a, Pb, pbase, wi, NW, rot, f);
     pbase += Pb;
   }
+}
+template <int PASS, typename V, int NW, int U, typename F>
+__device__ __forceinline__ void expand_tbl(const SpgemmArgs<V>& p, int64_t a0, int alen, int wi, unsigned char* tbl,
+                                           F&& f) {
+  esc_tbl_build<PASS, V, NW>(p, a0, alen, wi, tbl);
+  esc_tbl_gather<PASS, V, NW, U>(p, alen, wi, tbl, f);
 }
 
 // In-place exclusive scan of bc[0, NB) by the NW warps of the row (each thread a contiguous run
@@ -454,6 +497,15 @@ __host__ __device__ inline int64_t esc_staged_capacity(int pass, int64_t bytes) 
   return c < 65535 ? c : 65535;     // slot -> product indices are 16-bit
 }
 
+// exact shared-memory bytes of esc_row_staged's arrays for n products (without a reference table)
+template <typename V>
+__host__ __device__ inline int64_t esc_staged_bytes(int pass, int64_t n) {
+  int64_t NB = (n + kEscLambda - 1) / kEscLambda;
+  NB = (NB + 31) & ~(int64_t)31;
+  auto p16 = [](int64_t b) { return (b + 15) & ~(int64_t)15; };
+  return NB * 8 + p16(n * 4) + (pass == 1 ? p16(n * (int64_t)sizeof(V)) : 0) + p16(n * 2) + p16(n);
+}
+
 // rank of k among keys[idx[s .. en)] (keys < k); warp-uniform trip count as esc_rank
 __device__ __forceinline__ int esc_rank_ind(const uint32_t* keys, const uint16_t* idx, int s, int en, uint32_t k) {
   const int len = en - s;
@@ -474,7 +526,8 @@ __device__ __forceinline__ int esc_rank_ind(const uint32_t* keys, const uint16_t
 template <int NW, int PASS, typename V>
 __device__ __forceinline__ int esc_row_staged(const SpgemmArgs<V>& p, unsigned char* region, uint32_t region_bytes,
                                               int wi, int64_t a0, int alen, int n, int cnt, int32_t cmin,
-                                              int32_t cmax, int64_t cbase, int* red, const PreBatch<V>* pre = nullptr) {
+                                              int32_t cmax, int64_t cbase, int* red, const PreBatch<V>* pre = nullptr,
+                                              const unsigned char* ptbl = nullptr) {
   const int lane = lane_id();
   const int t = wi * 32 + lane;
   constexpr int T = NW * 32;
@@ -504,7 +557,7 @@ __device__ __forceinline__ int esc_row_staged(const SpgemmArgs<V>& p, unsigned c
     if (dups) dc[b] = 0;
   }
   unsigned char* tbl = jb + pad16((size_t)n);
-  const bool use_tbl = NW > 1 && kEscTable && (size_t)(tbl - region) + (size_t)esc_tbl_bytes<V>(alen) <= region_bytes;
+  const bool use_tbl = !ptbl && NW > 1 && kEscTable && (size_t)(tbl - region) + (size_t)esc_tbl_bytes<V>(alen) <= region_bytes;
   if (!use_tbl) esc_sync<NW>();     // (expand_tbl's barrier after the table build orders the clearing)
   // ---- G: gather (column, a*b) in product order; count the buckets --------------------------
   auto gather = [&](uint32_t col, V v, bool act, int pi) {
@@ -515,7 +568,9 @@ __device__ __forceinline__ int esc_row_staged(const SpgemmArgs<V>& p, unsigned c
       jb[pi] = (uint8_t)(j < 255 ? j : 255);
     }
   };
-  if (use_tbl)
+  if (ptbl)
+    esc_tbl_gather<PASS, V, NW, PASS == 0 ? 4 : 2>(p, alen, wi, ptbl, gather);   // table built by the caller
+  else if (use_tbl)
     expand_tbl<PASS, V, NW, PASS == 0 ? 4 : 2>(p, a0, alen, wi, tbl, gather);   // batches set up once per row
   else
     expand_esc<PASS, V, PASS == 0 ? 4 : 2>(p, a0, alen, wi, NW, gather, pre);

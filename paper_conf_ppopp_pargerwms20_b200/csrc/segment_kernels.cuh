@@ -190,6 +190,27 @@ __global__ void __launch_bounds__(kCfgThreads[kSegCfg], 1024 / kCfgThreads[kSegC
     count_path(p.paths, sg.dense == SEG_HASH ? SPECK_PATH_SEG_HASH : sg.dense == SEG_DENSE ? SPECK_PATH_SEG_DENSE
                                                                                          : SPECK_PATH_SEG_WINDOWS);
 
+  if (sg.dense == SEG_HASH && kEscStaged && p.esc >= 1) {
+    // counting sort of the segment (esc_row_staged): the clipped reference table goes to the
+    // end of the region, the products of the segment are counted from it; segments that do not
+    // fit (or have uneven buckets) take the ordered hash map below
+    constexpr uint32_t R = (uint32_t)kCfgMapBytes[CFG];
+    const int64_t tb = esc_tbl_bytes<V>(alen);
+    if (tb + 4096 <= (int64_t)R) {
+      const uint32_t toff = (uint32_t)(((int64_t)R - tb) & ~(int64_t)15);
+      unsigned char* tbl = smem + toff;
+      esc_tbl_build<1, V, NW>(p, a0, alen, warp_id(), tbl, true, lo, hi);
+      const int* tpb = EscTbl<V>(tbl, alen).pb;
+      int64_t n = 0;
+      for (int j = 0; j < (alen + 31) >> 5; ++j) n += tpb[j];
+      if (n > 0 && n <= 65535 && esc_staged_bytes<V>(1, n) <= (int64_t)toff) {
+        const int c = esc_row_staged<NW, 1, V>(p, smem, toff, warp_id(), a0, alen, (int)n, sg.cnt, (int32_t)lo,
+                                               (int32_t)(hi - 1), sg.out, reinterpret_cast<int*>(part), nullptr, tbl);
+        if (c >= 0) return;
+      }
+      __syncthreads();   // the hash map below reuses the region
+    }
+  }
   if (sg.dense == SEG_HASH) {
     uint32_t* keys = reinterpret_cast<uint32_t*>(smem);
     V* vals = reinterpret_cast<V*>(smem + num_val_offset<V>(CFG));
