@@ -69,9 +69,15 @@ struct SegPlanArgs {
   int split_max;           // >1: CTAs per candidate; rows with a kept bitmap split their A entries
                            //     over up to this many CTAs (C.val zeroed beforehand by the host)
 };
-constexpr int64_t kSplitProducts = 1 << 19;   // products per CTA of a split long row
+#ifndef SPECK_SPLIT_LOG2
+#define SPECK_SPLIT_LOG2 18     // C4 long_bitmap 2.95 -> 2.68 ms (profiles/r02/r02aq_*)
+#endif
+#ifndef SPECK_SPLIT_MAX_CAND
+#define SPECK_SPLIT_MAX_CAND 4096
+#endif
+constexpr int64_t kSplitProducts = (int64_t)1 << SPECK_SPLIT_LOG2;   // products per CTA of a split long row
 constexpr int kSplitPieces = 8;               // CTAs per candidate when splitting
-constexpr int64_t kSplitMaxCand = 4096;       // split only with few candidates (grid = candidates x pieces)
+constexpr int64_t kSplitMaxCand = SPECK_SPLIT_MAX_CAND;   // split only with few candidates (grid = candidates x pieces)
 
 // Long rows whose column range fits the shared-memory bitmap of k_long_bitmap.
 __device__ __forceinline__ bool bitmap_row(const SegPlanArgs& a, int32_t row) {
