@@ -77,6 +77,9 @@ constexpr uint32_t kEmptyKey = 0xFFFFFFFFu;
 #define SPECK_SYM_FILL 66
 #endif
 constexpr int kFillNum = SPECK_SYM_FILL;
+#ifndef SPECK_SYM_WARP_U
+#define SPECK_SYM_WARP_U 4   // product chunks in flight per symbolic warp row
+#endif
 #ifndef SPECK_SYM_REGION_X2
 #define SPECK_SYM_REGION_X2 8     // symbolic single-row regions: need * this / 2 slots (4x products: C5 symbolic 99 -> 91 ms)
 #endif

@@ -874,7 +874,10 @@ __device__ __forceinline__ int warp_row(const SpgemmArgs<V>& p, uint32_t* rk, V*
     if (g < 0) g = local_group_size(32, alen, warp_row_prods, warp_row_maxlen);
     expand_grouped<PASS, V>(p, a0, alen, 0, 1, g, ins);
   } else if (PASS == 0) {
-    expand_row<PASS, V, true, false, 2>(p, a0, alen, 0, 1, ins);
+    // symbolic warp rows by expand_esc too (REDUX owner search; the streamed shuffle binary search
+    // of expand_row measured slower once the probe was mask-based: C5 19.0 -> 18.3 ms, C2 A*P
+    // 1.39 -> 1.37 ms, profiles/r02/r02as_*)
+    expand_esc<PASS, V, SPECK_SYM_WARP_U>(p, a0, alen, 0, 1, ins);
   } else {
     expand_esc<PASS, V, SPECK_WARP_U>(p, a0, alen, 0, 1, ins, pre);
   }
